@@ -1,0 +1,274 @@
+/*
+ * pask.h -- C ABI of libpask.so, the B200-native hot path of PASK
+ * ("PASK: Cold Start Mitigation for Inference with Proactive and Selective
+ * Kernel Loading on GPUs", Huang, Du, Xiao, Zhang, DAC'25).  Citations are
+ * lines of /root/reference/PAPER.md ("PAPER.md:N") with their section.
+ *
+ * Problem statement (§III, Fig. 5): PASK "receives the lowered
+ * model (a sequence of n solutions) as input, and then proactively parses,
+ * loads, issues the DNN layer ... Upon absent solution, PASK seeks the
+ * opportunities to reuse the loaded solutions and organizes them based on
+ * their patterns".  Here the lowered model is a pask_graph, a "solution" is
+ * one kernel of the catalog below (PASK_K_*), and the library:
+ *   - plans (pask_plan / pask_load_model): Algorithm 1 EXECUTIONPLAN with the
+ *     categorical MRU cache (§III-B/C);
+ *   - loads proactively on a loader thread (PAPER.md:95, §III-A; :164 §III-D):
+ *     cuLibraryLoadData once, then cuLibraryGetKernel -> cuKernelGetFunction ->
+ *     cuFuncLoad per bound kernel, in first-use order;
+ *   - issues (pask_infer) on the caller's thread, each launch waiting only for
+ *     its own kernel's ready flag ("starts the kernels at the earliest feasible
+ *     time right after the loading").
+ *
+ * Conventions for every entry point:
+ *   - Returns PASK_OK (0) or a negative pask_status.  No C++ exception crosses
+ *     the ABI.  On error, pask_last_error() returns a thread-local message that
+ *     names the failing node / predicate / CUresult.
+ *   - There is no CPU fallback: a node with no applicable kernel fails with
+ *     PASK_EUNSUPPORTED; a driver failure returns PASK_ECUDA.
+ *   - Device memory (weights, every tensor, the workspace) is owned by the
+ *     caller and must stay alive until pask_destroy.  The library owns its host
+ *     structures, the CUlibrary/CUfunction handles, encoded CUtensorMaps and
+ *     the loader thread.
+ *   - A pask_ctx is not thread-safe: use one ctx per thread.
+ *   - The CUDA driver is loaded at run time (dlopen "libcuda.so.1"); the
+ *     host-only entry points (pask_plan, pask_workspace_bytes, pask_kernel_*)
+ *     work without a GPU.
+ */
+#ifndef PASK_H
+#define PASK_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PASK_VERSION 100
+
+typedef struct pask_ctx pask_ctx; /* opaque, library-owned */
+
+typedef enum {
+  PASK_OK = 0,
+  PASK_EINVAL = -1,      /* malformed graph / argument                                  */
+  PASK_EUNSUPPORTED = -2, /* a node's chosen solution s* is not applicable (no fallback)  */
+  PASK_ECUDA = -3,       /* driver call failed; message carries the CUresult name        */
+  PASK_ENOMEM = -4,      /* host allocation / workspace too small                        */
+  PASK_ESTATE = -5       /* call order violated (e.g. infer before load_model)           */
+} pask_status;
+
+typedef enum { PASK_BF16 = 0, PASK_F32 = 1 } pask_dtype;
+
+/* Memory order of a 4-D tensor with logical dims (n, h, w, c):
+ *   PASK_NCHW     : n, c, h, w (only the fp32 model input)
+ *   PASK_NHWC     : n, h, w, c (activations; c contiguous)
+ *   PASK_ROWMAJOR : a matrix of rows = n*h*w and cols = c (same bytes as NHWC) */
+typedef enum { PASK_NCHW = 0, PASK_NHWC = 1, PASK_ROWMAJOR = 2 } pask_layout;
+
+/* Operator classes of the lowered model ("PASK implements the
+ * reuse logic for the common convolution, pooling and activation primitives";
+ * PAPER.md:238 §VI extends it to GEMM). */
+typedef enum {
+  PASK_OP_LAYOUT = 0,   /* NCHW fp32 -> NHWC bf16, C zero-padded (PAPER.md:73 fn. 2)  */
+  PASK_OP_CONV2D = 1,   /* dense (groups = 1) or depthwise (groups = C = K)           */
+  PASK_OP_GEMM = 2,     /* batched C = act(A op(B) + bias + res)                      */
+  PASK_OP_POOL = 3,     /* max / avg, windowed or global                              */
+  PASK_OP_SOFTMAX = 4,  /* row softmax of scale * x                                   */
+  PASK_OP_LAYERNORM = 5 /* row LayerNorm, biased variance                             */
+} pask_op;
+
+/* Activations are fused epilogues of conv / GEMM (the activation primitive of
+ * PAPER.md:166; no standalone kernel). */
+typedef enum {
+  PASK_ACT_NONE = 0,
+  PASK_ACT_RELU = 1,
+  PASK_ACT_RELU6 = 2,
+  PASK_ACT_GELU_ERF = 3, /* 0.5 x (1 + erf(x / sqrt 2)) */
+  PASK_ACT_TANH = 4
+} pask_act;
+
+/* The kernel catalog ("solutions", PAPER.md:69, :73 fn. 2, :83 §II-B).  All of
+ * them live in ONE SASS-only code object embedded in libpask.so. */
+typedef enum {
+  PASK_K_LAYOUT = 0,     /* category (LAYOUT, f32, NCHW)                                */
+  PASK_K_CONV_IGEMM = 1, /* generic implicit-GEMM conv, tcgen05/TMEM; cat (CONV, bf16, NHWC) */
+  PASK_K_CONV_1X1 = 2,   /* specialised 1x1 s1 p0 conv (TMA-only A); cat (CONV, bf16, NHWC) */
+  PASK_K_CONV_DW = 3,    /* depthwise direct conv; cat (DWCONV, bf16, NHWC)             */
+  PASK_K_POOL = 4,       /* windowed max/avg pool; cat (POOL, bf16, NHWC)               */
+  PASK_K_POOL_GAVG = 5,  /* specialised global average pool; cat (POOL, bf16, NHWC)     */
+  PASK_K_GEMM = 6,       /* batched GEMM, tcgen05/TMEM; cat (GEMM, bf16, ROWMAJOR)      */
+  PASK_K_SOFTMAX = 7,    /* cat (SOFTMAX, bf16, ROWMAJOR)                               */
+  PASK_K_LAYERNORM = 8,  /* cat (LAYERNORM, bf16, ROWMAJOR)                             */
+  PASK_NUM_KERNELS = 9
+} pask_kernel_id;
+
+/* A tensor: logical dims (n, h, w, c), element type, memory order, and a
+ * caller-owned device pointer (16-byte aligned). */
+typedef struct {
+  int32_t dtype;  /* pask_dtype  */
+  int32_t layout; /* pask_layout */
+  int32_t n, h, w, c;
+  void *dptr;
+} pask_tensor;
+
+/* One lowered layer.  Fields not used by an op are ignored.
+ *
+ * LAYOUT   : in0 (NCHW f32, c <= out.c) -> out (NHWC bf16); channels c..out.c-1 = 0.
+ * CONV2D   : out[n,p,q,k] = act(bias[k] + res[n,p,q,k] +
+ *              sum_{c,r,s} in0[n, p*stride0 - pad0 + r*dil0, q*stride1 - pad1 + s*dil1, c]
+ *                          * w[k, r, s, c])                     (PAPER.md:83 patterns)
+ *            in0/out/res NHWC bf16; w KRSC bf16 (dense) or RSC bf16 (depthwise,
+ *            groups = C = K); bias fp32 [K] or NULL; res tensor index or -1.
+ * GEMM     : for b < batch, i < m, j < n:
+ *              C_b[i,j] = act( sum_{t<kk} A_b[i,t] * B_b[t,j] + bias[j] + R_b[i,j] )
+ *            A_b[i,t] = A[off_a + b*stride_a + i*lda + t]          (A = tensor in0)
+ *            B_b[t,j] = B[off_b + b*stride_b + j*ldb + t]  if trans_b (B stored [n][kk])
+ *                     = B[off_b + b*stride_b + t*ldb + j]  otherwise (B stored [kk][n])
+ *            B = w when w != NULL (weights), else tensor in1 (activation x activation)
+ *            C_b[i,j] = out[off_c + b*stride_c + i*ldc + j]; R uses res with the same
+ *            indexing.  All operands bf16; bias fp32 [n] or NULL.
+ * POOL     : pool_mode 0 = max (padding = -inf), 1 = avg (count_include_pad);
+ *            window (r, s), stride, pad; global_pool = 1 means window = (h, w).
+ * SOFTMAX  : rows = n*h*w of in0, cols = c: y = softmax(scale * x) per row.
+ * LAYERNORM: rows of in0: y = (x - mean) / sqrt(var + eps) * gamma + beta, var biased.
+ *
+ * solution: the statically chosen kernel s*_i carried by the lowered model
+ * (".mgx ... the determined optimal solutions for each layer"),
+ * or -1 to let the library apply its own static choice. */
+typedef struct {
+  int32_t op;       /* pask_op */
+  int32_t in0, in1, res, out; /* tensor indices; -1 = none */
+  const void *w;    /* device weights (see op)                  */
+  const float *bias, *gamma, *beta; /* device fp32 vectors or NULL */
+  int32_t k, r, s;
+  int32_t stride[2], pad[2], dil[2];
+  int32_t groups;
+  int32_t m, n, kk, batch, trans_b;
+  int64_t lda, ldb, ldc;
+  int64_t off_a, off_b, off_c;
+  int64_t stride_a, stride_b, stride_c;
+  int32_t pool_mode, count_include_pad, global_pool;
+  float eps, scale;
+  int32_t act;      /* pask_act */
+  int32_t solution; /* pask_kernel_id or -1 */
+} pask_node;
+
+typedef struct {
+  int32_t n_tensors;
+  const pask_tensor *tensors;
+  int32_t n_nodes;
+  const pask_node *nodes;
+  int32_t n_inputs;
+  const int32_t *inputs;  /* tensor indices fed by pask_infer(inputs)  */
+  int32_t n_outputs;
+  const int32_t *outputs; /* tensor indices read by pask_infer(outputs) */
+  void *workspace;        /* caller-owned device scratch, zero-filled before
+                             pask_load_model; >= pask_workspace_bytes()      */
+  uint64_t workspace_bytes;
+} pask_graph;
+
+typedef struct {
+  int32_t reuse;      /* 1 = Algorithm 1 reuse (PaSK); 0 = always load s* (PaSK-I / Baseline) */
+  int32_t search;     /* 0 = categorical MRU lists; 1 = naive scan (PaSK-R, :186) */
+  int32_t milestone;  /* m of PAPER.md:97; layers 1..m load s* unconditionally (default 0)    */
+  int32_t proactive;  /* 1 = loader thread; 0 = reactive load at first launch   */
+  int32_t pdl;        /* 1 = programmatic dependent launch between consecutive kernels        */
+  int32_t instrument; /* 1 = per-node CUDA events for gpu_busy_ns (perturbs timing)           */
+} pask_config;
+
+typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;
+
+typedef struct {
+  int32_t node;
+  int32_t desired_kernel; /* s*_i                                     */
+  int32_t bound_kernel;   /* s*_i or the substitute \hat{s}_i           */
+  int32_t how;            /* pask_how                                 */
+  int32_t lookups;        /* IsApplicable calls spent on this node    */
+} pask_binding;
+
+typedef struct {
+  int32_t n_nodes;
+  int32_t kernels_loaded;      /* distinct CUfunctions loaded for this model      */
+  int32_t code_objects_loaded; /* CUlibrary loads (1: single fatbin)              */
+  int32_t queries;             /* GETSUBSOLUTION calls (Alg. 1 l.6)               */
+  int32_t hits;                /* queries that returned a substitute              */
+  int32_t lookups;             /* IsApplicable calls inside queries              */
+  uint64_t code_bytes_loaded;  /* bytes of the code object handed to the driver  */
+  uint64_t plan_ns;            /* validation + problem extraction + Algorithm 1  */
+  uint64_t load_ns;            /* loader thread busy time (library + functions)  */
+  uint64_t load_exposed_ns;    /* issue thread blocked on not-yet-ready kernels  */
+  uint64_t issue_ns;           /* time inside cuLaunchKernelEx calls             */
+  uint64_t encode_ns;          /* CUtensorMap encoding + parameter packing        */
+  uint64_t gpu_span_ns;        /* first launch -> last kernel end, last inference */
+  uint64_t gpu_busy_ns;        /* sum of per-kernel times (instrument = 1 only)   */
+  uint64_t cold_wall_ns;       /* pask_load_model entry -> first inference done   */
+  uint64_t infer_count;
+  uint64_t launches;           /* kernel launches issued so far                   */
+} pask_stats_t;
+
+/* Library version (PASK_VERSION). */
+int pask_version(void);
+
+/* Create a context bound to the device's primary context (the one PyTorch
+ * uses) and start the (idle) loader thread.  cfg may be NULL for defaults
+ * {reuse 1, search 0, milestone 0, proactive 1, pdl 1, instrument 0}. */
+int pask_create(pask_ctx **ctx, int device, const pask_config *cfg);
+
+/* Host-only planning (no GPU needed): validate g, extract problems p_i, apply
+ * the static choice s*_i and Algorithm 1.  plan_out: caller-allocated
+ * [g->n_nodes]; stats_out (may be NULL) receives n_nodes, kernels_loaded
+ * (planned), queries, hits, lookups, plan_ns.  Deterministic: a pure function
+ * of (graph shapes, cfg). */
+int pask_plan(const pask_graph *g, const pask_config *cfg, pask_binding *plan_out,
+              pask_stats_t *stats_out);
+
+/* Bytes of zero-filled device workspace the graph needs (split-K partials and
+ * tile counters); host-only. */
+int pask_workspace_bytes(const pask_graph *g, uint64_t *bytes);
+
+/* Plan g (synchronously), hand the bound kernels to the loader thread in
+ * first-use order (asynchronously) and encode per-node launch parameters while
+ * loading proceeds.  plan_out may be NULL.  The graph arrays are copied; the
+ * device buffers they point to are not. */
+int pask_load_model(pask_ctx *ctx, const pask_graph *g, pask_binding *plan_out);
+
+/* Issue one inference on cuda_stream (a CUstream / cudaStream_t; NULL = legacy
+ * default stream).  inputs / outputs: device pointers, one per graph input /
+ * output, or NULL to use the tensors' bound dptr; a pointer different from the
+ * bound one rebinds that tensor (re-encoding the affected launch parameters).
+ * Blocks only while a needed kernel is still loading; returns after the last
+ * launch (asynchronous w.r.t. the GPU). */
+int pask_infer(pask_ctx *ctx, void *const *inputs, void *const *outputs, void *cuda_stream);
+
+/* End-to-end inference from host buffers: H2D copy of every graph input from
+ * host_inputs[i], pask_infer, D2H copy of every graph output into
+ * host_outputs[i], then stream synchronisation.  Pinned host memory is
+ * recommended; sizes follow the tensors' dims and dtype. */
+int pask_infer_host(pask_ctx *ctx, const void *const *host_inputs, void *const *host_outputs,
+                    void *cuda_stream);
+
+/* Wait for the last issued inference and finalise its timing statistics
+ * (gpu_span_ns; cold_wall_ns after the first inference). */
+int pask_sync(pask_ctx *ctx);
+
+/* Copy the statistics (host only; call pask_sync first for GPU times). */
+int pask_stats(const pask_ctx *ctx, pask_stats_t *out);
+
+/* Cross-check with the driver: *state = 1 if kernel_id's CUfunction is loaded
+ * in this context (cuFuncIsLoaded), 0 if not or never requested. */
+int pask_kernel_is_loaded(const pask_ctx *ctx, int32_t kernel_id, int32_t *state);
+
+/* Join the loader thread, unload the library and free host state. */
+int pask_destroy(pask_ctx *ctx);
+
+/* Thread-local description of the last error on this thread ("" if none). */
+const char *pask_last_error(void);
+
+/* Catalog introspection (host only). */
+int32_t pask_num_kernels(void);
+const char *pask_kernel_name(int32_t kernel_id);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* PASK_H */

@@ -1,0 +1,275 @@
+// HBM-bound kernels of the catalog: input layout (K10), depthwise conv (K5,
+// the DirectConv pattern of PAPER.md:83), pooling (K7), softmax
+// and LayerNorm (K11).  All use 128-bit vectors over the contiguous channel /
+// column dimension and fp32 arithmetic; reductions use warp shuffles.
+#pragma once
+#include "pask_params.h"
+#include "ptx.cuh"
+
+namespace pask {
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// ---------------------------------------------------------------- K10 layout
+// NCHW fp32 -> NHWC bf16 (RNE), channels c..c_out-1 zero.  One thread per
+// (pixel, 8-channel chunk): coalesced fp32 reads across pixels, one 16 B store.
+__device__ __forceinline__ void layout_body(const LayoutParams& p) {
+  pdl_wait();
+  pdl_launch_dependents();
+  const int chunks = p.c_out >> 3;
+  const int64_t hw = static_cast<int64_t>(p.h) * p.w;
+  const int64_t total = static_cast<int64_t>(p.n) * hw * chunks;
+  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < total;
+       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+    const int64_t pix = idx / chunks;
+    const int ch = static_cast<int>(idx - pix * chunks);
+    const int64_t n = pix / hw;
+    const int64_t off = pix - n * hw;
+    float f[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int c = ch * 8 + i;
+      f[i] = (c < p.c) ? __ldg(p.x + (n * p.c + c) * hw + off) : 0.f;
+    }
+    reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(f);
+  }
+}
+
+// ---------------------------------------------------------------- K7 pool
+// One thread per (output pixel, 8-channel chunk).  Max pads with -inf; avg
+// divides by the window or by the in-range count.
+__device__ __forceinline__ void pool_body(const PoolParams& p) {
+  pdl_wait();
+  pdl_launch_dependents();
+  const int chunks = p.C >> 3;
+  const int64_t total = static_cast<int64_t>(p.n) * p.P * p.Q * chunks;
+  const uint4* x = reinterpret_cast<const uint4*>(p.x);
+  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < total;
+       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+    int64_t t = idx;
+    const int ch = static_cast<int>(t % chunks);
+    t /= chunks;
+    const int q = static_cast<int>(t % p.Q);
+    t /= p.Q;
+    const int pp = static_cast<int>(t % p.P);
+    const int n = static_cast<int>(t / p.P);
+    float acc[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = p.mode == 0 ? -INFINITY : 0.f;
+    int cnt = 0;
+    const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
+    for (int r = 0; r < p.R; ++r) {
+      const int ih = ih0 + r;
+      if (ih < 0 || ih >= p.H) continue;
+      for (int s = 0; s < p.S; ++s) {
+        const int iw = iw0 + s;
+        if (iw < 0 || iw >= p.W) continue;
+        float f[8];
+        unpack_bf16x8(__ldg(x + ((static_cast<int64_t>(n) * p.H + ih) * p.W + iw) * chunks + ch), f);
+        ++cnt;
+        if (p.mode == 0) {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) acc[i] = fmaxf(acc[i], f[i]);
+        } else {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) acc[i] += f[i];
+        }
+      }
+    }
+    if (p.mode == 1) {
+      const float div = p.count_include_pad ? static_cast<float>(p.R * p.S) : static_cast<float>(cnt);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] = acc[i] / div;
+    }
+    reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(acc);
+  }
+}
+
+// Specialised global average pool (mean over H*W): one warp per (image,
+// 8-channel chunk) group of 32 chunks... one lane per chunk, pixels split over
+// the block's 4 warps, fp32 partial sums combined in shared memory.
+__device__ __forceinline__ void gavg_body(const PoolParams& p) {
+  __shared__ float red[4][32][8];
+  pdl_wait();
+  pdl_launch_dependents();
+  const int chunks = p.C >> 3;
+  const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;  // 4 warps
+  const int ch = blockIdx.x * 32 + lane;
+  const int n = blockIdx.y;
+  const int hw = p.H * p.W;
+  float acc[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) acc[i] = 0.f;
+  if (ch < chunks) {
+    const uint4* x = reinterpret_cast<const uint4*>(p.x) + static_cast<int64_t>(n) * hw * chunks + ch;
+    for (int px = wq; px < hw; px += 4) {
+      float f[8];
+      unpack_bf16x8(__ldg(x + static_cast<int64_t>(px) * chunks), f);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += f[i];
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) red[wq][lane][i] = acc[i];
+  __syncthreads();
+  if (wq == 0 && ch < chunks) {
+    const float inv = 1.f / static_cast<float>(hw);
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      acc[i] = (((red[0][lane][i] + red[1][lane][i]) + red[2][lane][i]) + red[3][lane][i]) * inv;
+    reinterpret_cast<uint4*>(p.y)[static_cast<int64_t>(n) * chunks + ch] = pack_bf16x8(acc);
+  }
+}
+
+// ---------------------------------------------------------------- K5 depthwise
+// One thread per (output pixel, 8-channel chunk); weights RSC so each tap is
+// one 16 B load of x and one of w; fused bias / residual / activation.
+__device__ __forceinline__ void dw_body(const DwParams& p) {
+  pdl_wait();
+  pdl_launch_dependents();
+  const int chunks = p.C >> 3;
+  const int64_t total = static_cast<int64_t>(p.n) * p.P * p.Q * chunks;
+  const uint4* x = reinterpret_cast<const uint4*>(p.x);
+  const uint4* w = reinterpret_cast<const uint4*>(p.w);
+  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < total;
+       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+    int64_t t = idx;
+    const int ch = static_cast<int>(t % chunks);
+    t /= chunks;
+    const int q = static_cast<int>(t % p.Q);
+    t /= p.Q;
+    const int pp = static_cast<int>(t % p.P);
+    const int n = static_cast<int>(t / p.P);
+    float acc[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = 0.f;
+    const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
+    for (int r = 0; r < p.R; ++r) {
+      const int ih = ih0 + r * p.dh;
+      if (ih < 0 || ih >= p.H) continue;
+      for (int s = 0; s < p.S; ++s) {
+        const int iw = iw0 + s * p.dw;
+        if (iw < 0 || iw >= p.W) continue;
+        float xf[8], wf[8];
+        unpack_bf16x8(__ldg(x + ((static_cast<int64_t>(n) * p.H + ih) * p.W + iw) * chunks + ch), xf);
+        unpack_bf16x8(__ldg(w + (r * p.S + s) * chunks + ch), wf);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = fmaf(xf[i], wf[i], acc[i]);
+      }
+    }
+    if (p.bias) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += __ldg(p.bias + ch * 8 + i);
+    }
+    if (p.res) {
+      float rf[8];
+      unpack_bf16x8(__ldg(reinterpret_cast<const uint4*>(p.res) + idx), rf);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += rf[i];
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = apply_act(acc[i], p.act);
+    reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(acc);
+  }
+}
+
+// ---------------------------------------------------------------- K11 softmax
+// One warp per row.  Pass 1: online max / sum of exp(scale*x - max) in fp32;
+// pass 2: write exp(scale*x - max) / sum as bf16.
+__device__ __forceinline__ void softmax_body(const RowParams& p) {
+  pdl_wait();
+  pdl_launch_dependents();
+  const int lane = threadIdx.x & 31;
+  const int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (row >= p.rows) return;
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
+  const bool vec = (p.cols & 7) == 0;
+  float m = -INFINITY, s = 0.f;
+  if (vec) {
+    for (int c = lane * 8; c < p.cols; c += 256) {
+      float f[8];
+      unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
+      float lm = m;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) lm = fmaxf(lm, f[i] * p.scale);
+      s *= __expf(m - lm);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) s += __expf(f[i] * p.scale - lm);
+      m = lm;
+    }
+  } else {
+    for (int c = lane; c < p.cols; c += 32) {
+      const float v = __bfloat162float(x[c]) * p.scale;
+      const float lm = fmaxf(m, v);
+      s = s * __expf(m - lm) + __expf(v - lm);
+      m = lm;
+    }
+  }
+  const float gm = warp_max(m);
+  s = (m == -INFINITY) ? 0.f : s * __expf(m - gm);
+  const float inv = 1.f / warp_sum(s);
+  if (vec) {
+    for (int c = lane * 8; c < p.cols; c += 256) {
+      float f[8];
+      unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) f[i] = __expf(f[i] * p.scale - gm) * inv;
+      *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f);
+    }
+  } else {
+    for (int c = lane; c < p.cols; c += 32)
+      y[c] = __float2bfloat16_rn(__expf(__bfloat162float(x[c]) * p.scale - gm) * inv);
+  }
+}
+
+// ---------------------------------------------------------------- K11 LayerNorm
+// One warp per row (cols % 8 == 0): mean, then biased variance of (x - mean)
+// (two passes over the row, fp32), then the affine transform.
+__device__ __forceinline__ void layernorm_body(const RowParams& p) {
+  pdl_wait();
+  pdl_launch_dependents();
+  const int lane = threadIdx.x & 31;
+  const int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (row >= p.rows) return;
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
+  float s = 0.f;
+  for (int c = lane * 8; c < p.cols; c += 256) {
+    float f[8];
+    unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) s += f[i];
+  }
+  const float mean = warp_sum(s) / static_cast<float>(p.cols);
+  float v = 0.f;
+  for (int c = lane * 8; c < p.cols; c += 256) {
+    float f[8];
+    unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float d = f[i] - mean;
+      v = fmaf(d, d, v);
+    }
+  }
+  const float rstd = rsqrtf(warp_sum(v) / static_cast<float>(p.cols) + p.eps);
+  for (int c = lane * 8; c < p.cols; c += 256) {
+    float f[8];
+    unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      f[i] = (f[i] - mean) * rstd * __ldg(p.gamma + c + i) + __ldg(p.beta + c + i);
+    *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f);
+  }
+}
+
+}  // namespace pask

@@ -1,0 +1,83 @@
+// Launch-parameter blocks shared by the host runtime (C++) and the sm_100a
+// kernels.  Each kernel takes exactly one of these by value as a
+// __grid_constant__ parameter; the CUtensorMaps inside are encoded on the host
+// at pask_load_model time (overlapping the proactive loads).
+#pragma once
+#include <cuda.h>
+#include <stdint.h>
+
+namespace pask {
+
+constexpr int kBM = 128;       // UMMA M (cta_group::1): one TMEM lane per tile row
+constexpr int kBK = 64;        // 64 bf16 = 128 B = one SWIZZLE_128B row
+constexpr int kGemmThreads = 192;  // warps 0-3 gather/epilogue, 4 TMA, 5 TMEM+MMA
+
+// A-operand source of the contraction kernel.
+enum AMode : int32_t {
+  A_TMA = 0,     // A is a plain K-major matrix: TMA tiled load (GEMM, 1x1 s1 p0 conv)
+  A_GATHER = 1,  // implicit im2col: cp.async gather with runtime pad/stride/dilation
+};
+
+struct alignas(64) GemmParams {
+  CUtensorMap tmap_a;  // A_TMA: 3-D {K, M, batch}, box {64, 128, 1}, SWIZZLE_128B
+  CUtensorMap tmap_b;  // K-major: {K, N, batch} box {64, BN, 1}; MN-major: {N, K, batch} box {64, 64, 1}
+  const void* x;       // A_GATHER: NHWC bf16 input
+  void* out;           // bf16 output (row i of tile at out + off_c + b*stride_c + i*ldc)
+  const void* res;     // bf16 residual, same indexing as out (nullable)
+  const float* bias;   // fp32 [N] (nullable)
+  float* ws_partial;   // split-K fp32 partial tiles
+  uint32_t* ws_counter;  // split-K arrival counters (self-resetting)
+  int64_t ldc, off_c, stride_c;
+  int32_t M, N, K, batch;
+  int32_t num_kb;        // ceil(K / 64)
+  int32_t kb_per_split;  // k-blocks per split
+  int32_t splits;        // grid.z = batch * splits
+  int32_t bn;            // N tile: 16..256, multiple of 16
+  int32_t stages;        // smem pipeline depth
+  int32_t a_mode;        // AMode
+  int32_t b_major;       // 0 K-major, 1 MN-major
+  int32_t act;           // pask_act
+  int32_t m_tiles, n_tiles;
+  // implicit-GEMM geometry (A_GATHER): input [n][H][W][C], output pixel m -> (n, p, q)
+  int32_t H, W, C, P, Q, R, S;
+  int32_t sh, sw, ph, pw, dh, dw;
+  uint32_t idesc;      // tcgen05 instruction descriptor (kind::f16, bf16 x bf16 -> f32)
+  uint32_t tmem_cols;  // power of two >= max(32, bn)
+  uint32_t smem_bytes;
+};
+
+struct alignas(16) LayoutParams {
+  const float* x;  // NCHW fp32
+  void* y;         // NHWC bf16, c_out channels (c_out % 8 == 0)
+  int32_t n, c, h, w, c_out;
+};
+
+struct alignas(16) PoolParams {
+  const void* x;  // NHWC bf16 [n][H][W][C]
+  void* y;        // NHWC bf16 [n][P][Q][C]
+  int32_t n, H, W, C, P, Q, R, S, sh, sw, ph, pw;
+  int32_t mode;   // 0 max, 1 avg
+  int32_t count_include_pad;
+};
+
+struct alignas(16) DwParams {
+  const void* x;       // NHWC bf16 [n][H][W][C]
+  const void* w;       // RSC bf16 [R][S][C]
+  const float* bias;   // [C] or null
+  const void* res;     // NHWC bf16 [n][P][Q][C] or null
+  void* y;             // NHWC bf16 [n][P][Q][C]
+  int32_t n, H, W, C, P, Q, R, S, sh, sw, ph, pw, dh, dw;
+  int32_t act;
+};
+
+struct alignas(16) RowParams {
+  const void* x;  // bf16 [rows][cols]
+  void* y;        // bf16 [rows][cols]
+  const float* gamma;
+  const float* beta;
+  int32_t rows, cols;
+  float scale;  // softmax
+  float eps;    // layernorm
+};
+
+}  // namespace pask

@@ -1,0 +1,48 @@
+// CUDA driver API resolved at run time (dlopen("libcuda.so.1") +
+// cuGetProcAddress), so libpask.so loads on machines without a GPU driver
+// (the host-only planner entry points then still work) and so tests can
+// substitute a fake driver table for the loader / issuer logic.
+#pragma once
+#include <cuda.h>
+
+namespace pask {
+
+struct Driver {
+#define PASK_DRV_FN(name) decltype(&::name) name = nullptr;
+  PASK_DRV_FN(cuInit)
+  PASK_DRV_FN(cuGetErrorName)
+  PASK_DRV_FN(cuDeviceGet)
+  PASK_DRV_FN(cuDeviceGetAttribute)
+  PASK_DRV_FN(cuDevicePrimaryCtxRetain)
+  PASK_DRV_FN(cuDevicePrimaryCtxRelease)
+  PASK_DRV_FN(cuCtxGetCurrent)
+  PASK_DRV_FN(cuCtxSetCurrent)
+  PASK_DRV_FN(cuLibraryLoadData)
+  PASK_DRV_FN(cuLibraryUnload)
+  PASK_DRV_FN(cuLibraryGetKernel)
+  PASK_DRV_FN(cuKernelGetFunction)
+  PASK_DRV_FN(cuFuncLoad)
+  PASK_DRV_FN(cuFuncIsLoaded)
+  PASK_DRV_FN(cuFuncSetAttribute)
+  PASK_DRV_FN(cuLaunchKernelEx)
+  PASK_DRV_FN(cuTensorMapEncodeTiled)
+  PASK_DRV_FN(cuEventCreate)
+  PASK_DRV_FN(cuEventDestroy)
+  PASK_DRV_FN(cuEventRecord)
+  PASK_DRV_FN(cuEventSynchronize)
+  PASK_DRV_FN(cuEventElapsedTime)
+  PASK_DRV_FN(cuMemcpyHtoDAsync)
+  PASK_DRV_FN(cuMemcpyDtoHAsync)
+  PASK_DRV_FN(cuStreamSynchronize)
+#undef PASK_DRV_FN
+  bool ok = false;
+};
+
+// Resolve the driver once (thread-safe).  Returns nullptr and sets *why when
+// libcuda is unavailable.
+const Driver* driver(const char** why);
+
+// Tests: replace the resolved driver table (nullptr restores the real one).
+void driver_override(const Driver* fake);
+
+}  // namespace pask

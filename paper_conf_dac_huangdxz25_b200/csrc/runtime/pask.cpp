@@ -1,0 +1,689 @@
+// libpask.so: the C ABI of include/pask.h.
+//
+// Threads (§III-A "PASK spawns two extra host threads to handle
+// code loading and kernel issuing"; :164 §III-D SPSC channels):
+//   * caller thread = parser + planner (pask_load_model) and issuer (pask_infer);
+//   * one loader thread per context, fed a FIFO of kernel ids in first-use order
+//     (single producer: the planner; single consumer: the loader), publishing each
+//     loaded CUfunction through a per-kernel atomic ready flag that the issuer
+//     acquires right before the launch that needs it.
+#include <immintrin.h>
+#include <pthread.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstdio>
+#include <cstdlib>
+#include <deque>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../kernels/pask_params.h"
+#include "driver.h"
+#include "plan.h"
+
+#define PASK_API extern "C" __attribute__((visibility("default")))
+
+extern "C" const unsigned char pask_fatbin_start[];
+extern "C" const unsigned char pask_fatbin_end[];
+
+namespace pask {
+
+namespace {
+
+thread_local std::string t_err;
+
+int set_err(int code, const std::string& m) {
+  t_err = m;
+  return code;
+}
+
+uint64_t now_ns() {
+  return static_cast<uint64_t>(
+      std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
+          .count());
+}
+
+union alignas(64) AnyParams {
+  GemmParams g;
+  LayoutParams l;
+  PoolParams p;
+  DwParams d;
+  RowParams r;
+};
+
+struct Launch {
+  int32_t kernel = -1;
+  unsigned grid[3] = {1, 1, 1};
+  unsigned block[3] = {1, 1, 1};
+  unsigned smem = 0;
+  std::unique_ptr<AnyParams> params;
+};
+
+bool is_gemm_kernel(int32_t k) {
+  return k == PASK_K_CONV_IGEMM || k == PASK_K_CONV_1X1 || k == PASK_K_GEMM;
+}
+
+}  // namespace
+
+struct Ctx {
+  const Driver* d = nullptr;
+  int device = 0;
+  CUcontext cuctx = nullptr;
+  pask_config cfg{};
+
+  // ---- loader (proactive code loading)
+  std::thread loader;
+  std::mutex mu;
+  std::condition_variable cv;
+  std::deque<int32_t> fifo;
+  bool stop = false;
+  std::mutex lib_mu;  // serialises library/function loads (loader vs reactive issuer)
+  CUlibrary lib = nullptr;
+  std::atomic<int32_t> ready[PASK_NUM_KERNELS];
+  CUfunction fn[PASK_NUM_KERNELS] = {};
+  CUresult kerr[PASK_NUM_KERNELS] = {};
+  bool requested[PASK_NUM_KERNELS] = {};
+  std::atomic<uint64_t> load_ns{0};
+  std::atomic<int32_t> code_objects{0};
+  std::atomic<uint64_t> code_bytes{0};
+  std::atomic<int32_t> kernels_loaded{0};
+
+  // ---- model
+  bool have_model = false;
+  std::vector<pask_tensor> tensors;
+  std::vector<pask_node> nodes;
+  std::vector<int32_t> inputs, outputs;
+  void* ws = nullptr;
+  uint64_t ws_bytes = 0;
+  std::vector<Problem> probs;
+  PlanResult plan;
+  std::vector<Launch> launches;
+
+  // ---- timing / stats
+  pask_stats_t st{};
+  uint64_t t_entry = 0;
+  bool first_done = false;
+  bool pending = false;
+  CUevent ev0 = nullptr, ev1 = nullptr;
+  std::vector<CUevent> node_ev;
+
+  Ctx() {
+    for (auto& r : ready) r.store(0);
+  }
+};
+
+namespace {
+
+std::string cu_err(const Driver* d, CUresult r, const char* what) {
+  const char* name = nullptr;
+  if (d && d->cuGetErrorName) d->cuGetErrorName(r, &name);
+  return std::string(what) + " failed: " + (name ? name : "CUDA_ERROR_?") + " (" + std::to_string(r) + ")";
+}
+
+// Load one catalog kernel into the context: library once, then
+// cuLibraryGetKernel -> cuKernelGetFunction -> cuFuncLoad (A13 of SURVEY.md §2).
+void load_kernel(Ctx* c, int32_t k) {
+  std::lock_guard<std::mutex> g(c->lib_mu);
+  if (c->ready[k].load(std::memory_order_acquire) != 0) return;
+  const uint64_t t0 = now_ns();
+  const Driver* d = c->d;
+  CUresult r = CUDA_SUCCESS;
+  if (!c->lib) {
+    const size_t bytes = static_cast<size_t>(pask_fatbin_end - pask_fatbin_start);
+    r = d->cuLibraryLoadData(&c->lib, pask_fatbin_start, nullptr, nullptr, 0, nullptr, nullptr, 0);
+    if (r == CUDA_SUCCESS) {
+      c->code_objects.fetch_add(1);
+      c->code_bytes.fetch_add(bytes);
+    }
+  }
+  CUkernel kern = nullptr;
+  CUfunction f = nullptr;
+  if (r == CUDA_SUCCESS) r = d->cuLibraryGetKernel(&kern, c->lib, catalog(k).name);
+  if (r == CUDA_SUCCESS) r = d->cuKernelGetFunction(&f, kern);
+  if (r == CUDA_SUCCESS) r = d->cuFuncLoad(f);
+  if (r == CUDA_SUCCESS && is_gemm_kernel(k))
+    r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 227 * 1024);
+  c->fn[k] = f;
+  c->kerr[k] = r;
+  if (r == CUDA_SUCCESS) c->kernels_loaded.fetch_add(1);
+  c->load_ns.fetch_add(now_ns() - t0);
+  c->ready[k].store(r == CUDA_SUCCESS ? 1 : -1, std::memory_order_release);
+}
+
+void loader_main(Ctx* c) {
+  pthread_setname_np(pthread_self(), "pask-loader");
+  c->d->cuCtxSetCurrent(c->cuctx);
+  for (;;) {
+    int32_t k;
+    {
+      std::unique_lock<std::mutex> lk(c->mu);
+      c->cv.wait(lk, [&] { return c->stop || !c->fifo.empty(); });
+      if (c->stop && c->fifo.empty()) return;
+      k = c->fifo.front();
+      c->fifo.pop_front();
+    }
+    load_kernel(c, k);
+  }
+}
+
+// ------------------------------------------------------------------ tensor maps
+int encode_3d(Ctx* c, CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1, uint64_t d2,
+              uint64_t s1_bytes, uint64_t s2_bytes, uint32_t b0, uint32_t b1, std::string* err) {
+  if (d2 <= 1) s2_bytes = s1_bytes * d1;
+  cuuint64_t dims[3] = {d0, d1, std::max<uint64_t>(d2, 1)};
+  cuuint64_t strides[2] = {s1_bytes, s2_bytes};
+  cuuint32_t box[3] = {b0, b1, 1};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = c->d->cuTensorMapEncodeTiled(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims,
+                                            strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    *err = cu_err(c->d, r, "cuTensorMapEncodeTiled");
+    return PASK_ECUDA;
+  }
+  return PASK_OK;
+}
+
+uint32_t make_idesc(int bn, int b_major) {
+  uint32_t d = 0;
+  d |= 1u << 4;                              // D format f32
+  d |= 1u << 7;                              // A bf16
+  d |= 1u << 10;                             // B bf16
+  d |= static_cast<uint32_t>(b_major) << 16;  // B major (A is always K-major)
+  d |= static_cast<uint32_t>(bn >> 3) << 17;  // N >> 3
+  d |= static_cast<uint32_t>(128 >> 4) << 24;  // M >> 4
+  return d;
+}
+
+unsigned grid_1d(int64_t total, int threads) {
+  int64_t b = (total + threads - 1) / threads;
+  if (b < 1) b = 1;
+  if (b > 148 * 16) b = 148 * 16;  // grid-stride beyond 16 waves of 1 CTA/SM
+  return static_cast<unsigned>(b);
+}
+
+// Build the launch (grid, block, smem, parameter block) of node i for its bound kernel.
+int lower_node(Ctx* c, int32_t i, std::string* err) {
+  const pask_node& nd = c->nodes[i];
+  const Problem& p = c->probs[i];
+  Launch& L = c->launches[i];
+  L.kernel = c->plan.bindings[i].bound_kernel;
+  if (!L.params) L.params.reset(new AnyParams);
+  memset(L.params.get(), 0, sizeof(AnyParams));
+  const pask_tensor& x = c->tensors[nd.in0];
+  const pask_tensor& y = c->tensors[nd.out];
+  const void* res = nd.res >= 0 ? c->tensors[nd.res].dptr : nullptr;
+  L.block[0] = 256;
+  L.block[1] = L.block[2] = 1;
+  L.grid[1] = L.grid[2] = 1;
+  L.smem = 0;
+  switch (L.kernel) {
+    case PASK_K_LAYOUT: {
+      LayoutParams& q = L.params->l;
+      q.x = static_cast<const float*>(x.dptr);
+      q.y = y.dptr;
+      q.n = p.n; q.c = p.c; q.h = p.h; q.w = p.w; q.c_out = p.k;
+      L.grid[0] = grid_1d(static_cast<int64_t>(p.n) * p.h * p.w * (p.k / 8), 256);
+      return PASK_OK;
+    }
+    case PASK_K_CONV_DW: {
+      DwParams& q = L.params->d;
+      q.x = x.dptr; q.w = nd.w; q.bias = nd.bias; q.res = res; q.y = y.dptr;
+      q.n = p.n; q.H = p.h; q.W = p.w; q.C = p.c; q.P = p.p; q.Q = p.q; q.R = p.r; q.S = p.s;
+      q.sh = p.stride_h; q.sw = p.stride_w; q.ph = p.pad_h; q.pw = p.pad_w; q.dh = p.dil_h; q.dw = p.dil_w;
+      q.act = nd.act;
+      L.grid[0] = grid_1d(static_cast<int64_t>(p.n) * p.p * p.q * (p.c / 8), 256);
+      return PASK_OK;
+    }
+    case PASK_K_POOL:
+    case PASK_K_POOL_GAVG: {
+      PoolParams& q = L.params->p;
+      q.x = x.dptr; q.y = y.dptr;
+      q.n = p.n; q.H = p.h; q.W = p.w; q.C = p.c; q.P = p.p; q.Q = p.q; q.R = p.r; q.S = p.s;
+      q.sh = p.stride_h; q.sw = p.stride_w; q.ph = p.pad_h; q.pw = p.pad_w;
+      q.mode = p.pool_mode; q.count_include_pad = nd.count_include_pad;
+      if (L.kernel == PASK_K_POOL_GAVG) {
+        L.block[0] = 128;
+        L.grid[0] = static_cast<unsigned>((p.c / 8 + 31) / 32);
+        L.grid[1] = static_cast<unsigned>(p.n);
+      } else {
+        L.grid[0] = grid_1d(static_cast<int64_t>(p.n) * p.p * p.q * (p.c / 8), 256);
+      }
+      return PASK_OK;
+    }
+    case PASK_K_SOFTMAX:
+    case PASK_K_LAYERNORM: {
+      RowParams& q = L.params->r;
+      q.x = x.dptr; q.y = y.dptr; q.gamma = nd.gamma; q.beta = nd.beta;
+      q.rows = p.rows; q.cols = p.cols; q.scale = nd.scale; q.eps = nd.eps;
+      L.grid[0] = static_cast<unsigned>((p.rows + 7) / 8);
+      return PASK_OK;
+    }
+    case PASK_K_CONV_IGEMM:
+    case PASK_K_CONV_1X1:
+    case PASK_K_GEMM: {
+      GemmParams& q = L.params->g;
+      int32_t M, N, K, batch, b_major;
+      contraction_shape(p, nd, &M, &N, &K, &batch, &b_major);
+      const GemmTiling t = gemm_tiling(M, N, K, batch, b_major);
+      q.M = M; q.N = N; q.K = K; q.batch = batch;
+      q.num_kb = t.num_kb; q.kb_per_split = t.kb_per_split; q.splits = t.splits;
+      q.bn = t.bn; q.stages = t.stages; q.b_major = b_major; q.act = nd.act;
+      q.m_tiles = t.m_tiles; q.n_tiles = t.n_tiles;
+      q.idesc = make_idesc(t.bn, b_major);
+      q.tmem_cols = t.tmem_cols;
+      q.smem_bytes = t.smem_bytes;
+      q.out = y.dptr; q.res = res; q.bias = nd.bias;
+      const uint64_t cnt_region = (t.ws_counter_bytes + 255) / 256 * 256;
+      if (t.splits > 1) {
+        if (!c->ws || c->ws_bytes < cnt_region + t.ws_partial_bytes) {
+          *err = "node " + std::to_string(i) + ": workspace too small (see pask_workspace_bytes)";
+          return PASK_ENOMEM;
+        }
+        q.ws_counter = static_cast<uint32_t*>(c->ws);
+        q.ws_partial = reinterpret_cast<float*>(static_cast<char*>(c->ws) + cnt_region);
+      }
+      int rc;
+      if (p.op == OC_CONV) {
+        q.ldc = p.k; q.off_c = 0; q.stride_c = 0;
+        const bool plain = (p.r == 1 && p.s == 1 && p.stride_h == 1 && p.stride_w == 1 && p.pad_h == 0 &&
+                            p.pad_w == 0);
+        q.a_mode = (L.kernel == PASK_K_CONV_1X1 || plain) ? A_TMA : A_GATHER;
+        q.x = x.dptr;
+        q.H = p.h; q.W = p.w; q.C = p.c; q.P = p.p; q.Q = p.q; q.R = p.r; q.S = p.s;
+        q.sh = p.stride_h; q.sw = p.stride_w; q.ph = p.pad_h; q.pw = p.pad_w; q.dh = p.dil_h; q.dw = p.dil_w;
+        if (q.a_mode == A_TMA) {
+          rc = encode_3d(c, &q.tmap_a, x.dptr, static_cast<uint64_t>(K), static_cast<uint64_t>(M), 1,
+                         static_cast<uint64_t>(p.c) * 2, 0, 64, 128, err);
+          if (rc) return rc;
+        }
+        // weights KRSC = [N][K] K-major
+        rc = encode_3d(c, &q.tmap_b, nd.w, static_cast<uint64_t>(K), static_cast<uint64_t>(N), 1,
+                       static_cast<uint64_t>(K) * 2, 0, 64, static_cast<uint32_t>(t.bn), err);
+        if (rc) return rc;
+      } else {
+        q.ldc = nd.ldc; q.off_c = nd.off_c; q.stride_c = nd.stride_c;
+        q.a_mode = A_TMA;
+        const char* abase = static_cast<const char*>(x.dptr) + nd.off_a * 2;
+        rc = encode_3d(c, &q.tmap_a, abase, static_cast<uint64_t>(K), static_cast<uint64_t>(M),
+                       static_cast<uint64_t>(batch), static_cast<uint64_t>(nd.lda) * 2,
+                       static_cast<uint64_t>(nd.stride_a) * 2, 64, 128, err);
+        if (rc) return rc;
+        const void* bsrc = nd.w ? nd.w : c->tensors[nd.in1].dptr;
+        const char* bbase = static_cast<const char*>(bsrc) + nd.off_b * 2;
+        if (b_major == 0)
+          rc = encode_3d(c, &q.tmap_b, bbase, static_cast<uint64_t>(K), static_cast<uint64_t>(N),
+                         static_cast<uint64_t>(batch), static_cast<uint64_t>(nd.ldb) * 2,
+                         static_cast<uint64_t>(nd.stride_b) * 2, 64, static_cast<uint32_t>(t.bn), err);
+        else
+          rc = encode_3d(c, &q.tmap_b, bbase, static_cast<uint64_t>(N), static_cast<uint64_t>(K),
+                         static_cast<uint64_t>(batch), static_cast<uint64_t>(nd.ldb) * 2,
+                         static_cast<uint64_t>(nd.stride_b) * 2, 64, 64, err);
+        if (rc) return rc;
+      }
+      L.block[0] = kGemmThreads;
+      L.grid[0] = static_cast<unsigned>(t.m_tiles);
+      L.grid[1] = static_cast<unsigned>(t.n_tiles);
+      L.grid[2] = static_cast<unsigned>(batch * t.splits);
+      L.smem = t.smem_bytes;
+      return PASK_OK;
+    }
+  }
+  *err = "node " + std::to_string(i) + ": no lowering for kernel";
+  return PASK_EINVAL;
+}
+
+int plan_graph(const pask_graph* g, const pask_config& cfg, std::vector<Problem>* probs, PlanResult* plan) {
+  std::string err;
+  int rc = extract_problems(g, probs, &err);
+  if (rc) return set_err(rc, err);
+  std::vector<int32_t> desired(probs->size());
+  for (size_t i = 0; i < probs->size(); ++i) {
+    const int32_t sol = g->nodes[i].solution;
+    desired[i] = (sol >= 0) ? sol : static_choice((*probs)[i]);
+  }
+  rc = execution_plan(*probs, desired, cfg, plan, &err);
+  if (rc) return set_err(rc, err);
+  return PASK_OK;
+}
+
+int wait_kernel(Ctx* c, int32_t k) {
+  int32_t s = c->ready[k].load(std::memory_order_acquire);
+  if (s == 0) {
+    const uint64_t t0 = now_ns();
+    if (!c->cfg.proactive) {
+      load_kernel(c, k);  // reactive: load at launch, on the issue thread (A1 baseline)
+    } else {
+      if (!c->requested[k]) {  // not planned for loading (e.g. rebinding) -> queue it now
+        std::lock_guard<std::mutex> lk(c->mu);
+        c->requested[k] = true;
+        c->fifo.push_back(k);
+        c->cv.notify_one();
+      }
+      while ((s = c->ready[k].load(std::memory_order_acquire)) == 0) _mm_pause();
+    }
+    c->st.load_exposed_ns += now_ns() - t0;
+    s = c->ready[k].load(std::memory_order_acquire);
+  }
+  if (s < 0)
+    return set_err(PASK_ECUDA, cu_err(c->d, c->kerr[k], (std::string("loading ") + catalog(k).name).c_str()));
+  return PASK_OK;
+}
+
+int rebind(Ctx* c, int32_t tidx, void* ptr) {
+  if (c->tensors[tidx].dptr == ptr) return PASK_OK;
+  c->tensors[tidx].dptr = ptr;
+  std::string err;
+  for (size_t i = 0; i < c->nodes.size(); ++i) {
+    const pask_node& nd = c->nodes[i];
+    if (nd.in0 == tidx || nd.in1 == tidx || nd.res == tidx || nd.out == tidx) {
+      int rc = lower_node(c, static_cast<int32_t>(i), &err);
+      if (rc) return set_err(rc, err);
+    }
+  }
+  return PASK_OK;
+}
+
+size_t tensor_bytes(const pask_tensor& t) {
+  return static_cast<size_t>(t.n) * t.h * t.w * t.c * (t.dtype == PASK_F32 ? 4 : 2);
+}
+
+}  // namespace
+}  // namespace pask
+
+using namespace pask;
+
+struct pask_ctx : pask::Ctx {};
+
+// ====================================================================== API
+PASK_API int pask_version(void) { return PASK_VERSION; }
+
+PASK_API const char* pask_last_error(void) { return t_err.c_str(); }
+
+PASK_API int32_t pask_num_kernels(void) { return PASK_NUM_KERNELS; }
+
+PASK_API const char* pask_kernel_name(int32_t id) {
+  if (id < 0 || id >= PASK_NUM_KERNELS) return "";
+  return catalog(id).name;
+}
+
+PASK_API int pask_plan(const pask_graph* g, const pask_config* cfg, pask_binding* plan_out,
+                       pask_stats_t* stats_out) {
+  t_err.clear();
+  const uint64_t t0 = now_ns();
+  pask_config c = cfg ? *cfg : default_config();
+  std::vector<Problem> probs;
+  PlanResult plan;
+  int rc = plan_graph(g, c, &probs, &plan);
+  if (rc) return rc;
+  if (plan_out) memcpy(plan_out, plan.bindings.data(), plan.bindings.size() * sizeof(pask_binding));
+  if (stats_out) {
+    memset(stats_out, 0, sizeof(*stats_out));
+    stats_out->n_nodes = g->n_nodes;
+    stats_out->kernels_loaded = static_cast<int32_t>(plan.loaded.size());
+    stats_out->queries = plan.queries;
+    stats_out->hits = plan.hits;
+    stats_out->lookups = plan.lookups;
+    stats_out->plan_ns = now_ns() - t0;
+  }
+  return PASK_OK;
+}
+
+PASK_API int pask_workspace_bytes(const pask_graph* g, uint64_t* bytes) {
+  t_err.clear();
+  if (!bytes) return set_err(PASK_EINVAL, "bytes is null");
+  std::vector<Problem> probs;
+  std::string err;
+  int rc = extract_problems(g, &probs, &err);
+  if (rc) return set_err(rc, err);
+  uint64_t need = 0;
+  for (size_t i = 0; i < probs.size(); ++i) {
+    int32_t M, N, K, batch, bm;
+    if (!contraction_shape(probs[i], g->nodes[i], &M, &N, &K, &batch, &bm)) continue;
+    const GemmTiling t = gemm_tiling(M, N, K, batch, bm);
+    if (t.splits > 1) need = std::max(need, (t.ws_counter_bytes + 255) / 256 * 256 + t.ws_partial_bytes);
+  }
+  *bytes = need;
+  return PASK_OK;
+}
+
+PASK_API int pask_create(pask_ctx** out, int device, const pask_config* cfg) {
+  t_err.clear();
+  if (!out) return set_err(PASK_EINVAL, "ctx out-pointer is null");
+  *out = nullptr;
+  const char* why = "";
+  const Driver* d = driver(&why);
+  if (!d) return set_err(PASK_ECUDA, std::string("CUDA driver unavailable: ") + why);
+  CUresult r = d->cuInit(0);
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuInit"));
+  std::unique_ptr<pask_ctx> c(new pask_ctx);
+  c->d = d;
+  c->device = device;
+  c->cfg = cfg ? *cfg : default_config();
+  CUcontext cur = nullptr;
+  d->cuCtxGetCurrent(&cur);
+  if (!cur) {
+    CUdevice dev;
+    r = d->cuDeviceGet(&dev, device);
+    if (r == CUDA_SUCCESS) r = d->cuDevicePrimaryCtxRetain(&cur, dev);
+    if (r == CUDA_SUCCESS) r = d->cuCtxSetCurrent(cur);
+    if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "primary context"));
+  }
+  c->cuctx = cur;
+  r = d->cuEventCreate(&c->ev0, CU_EVENT_DEFAULT);
+  if (r == CUDA_SUCCESS) r = d->cuEventCreate(&c->ev1, CU_EVENT_DEFAULT);
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuEventCreate"));
+  pask_ctx* raw = c.get();
+  raw->loader = std::thread(loader_main, raw);
+  *out = c.release();
+  return PASK_OK;
+}
+
+PASK_API int pask_load_model(pask_ctx* c, const pask_graph* g, pask_binding* plan_out) {
+  t_err.clear();
+  if (!c || !g) return set_err(PASK_EINVAL, "null ctx or graph");
+  if (c->have_model) return set_err(PASK_ESTATE, "a model is already loaded in this context");
+  c->t_entry = now_ns();
+  // ---- parse + plan (Algorithm 1)
+  int rc = plan_graph(g, c->cfg, &c->probs, &c->plan);
+  if (rc) return rc;
+  const uint64_t t_plan = now_ns();
+  // ---- proactive loading: hand the bound kernels to the loader, first-use order
+  if (c->cfg.proactive) {
+    std::lock_guard<std::mutex> lk(c->mu);
+    for (const pask_binding& b : c->plan.bindings) {
+      const int32_t k = b.bound_kernel;
+      if (!c->requested[k]) {
+        c->requested[k] = true;
+        c->fifo.push_back(k);
+      }
+    }
+    c->cv.notify_one();
+  }
+  // ---- copy the graph and lower every node while loading proceeds
+  c->tensors.assign(g->tensors, g->tensors + g->n_tensors);
+  c->nodes.assign(g->nodes, g->nodes + g->n_nodes);
+  c->inputs.assign(g->inputs, g->inputs + g->n_inputs);
+  c->outputs.assign(g->outputs, g->outputs + g->n_outputs);
+  for (int32_t t : c->inputs)
+    if (t < 0 || t >= g->n_tensors) return set_err(PASK_EINVAL, "graph input index out of range");
+  for (int32_t t : c->outputs)
+    if (t < 0 || t >= g->n_tensors) return set_err(PASK_EINVAL, "graph output index out of range");
+  c->ws = g->workspace;
+  c->ws_bytes = g->workspace_bytes;
+  c->launches.clear();
+  c->launches.resize(g->n_nodes);
+  std::string err;
+  for (int32_t i = 0; i < g->n_nodes; ++i) {
+    rc = lower_node(c, i, &err);
+    if (rc) return set_err(rc, err);
+  }
+  if (c->cfg.instrument) {
+    c->node_ev.resize(2 * g->n_nodes);
+    for (auto& e : c->node_ev) {
+      CUresult r = c->d->cuEventCreate(&e, CU_EVENT_DEFAULT);
+      if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(c->d, r, "cuEventCreate"));
+    }
+  }
+  const uint64_t t_enc = now_ns();
+  memset(&c->st, 0, sizeof(c->st));
+  c->st.n_nodes = g->n_nodes;
+  c->st.queries = c->plan.queries;
+  c->st.hits = c->plan.hits;
+  c->st.lookups = c->plan.lookups;
+  c->st.plan_ns = t_plan - c->t_entry;
+  c->st.encode_ns = t_enc - t_plan;
+  if (plan_out) memcpy(plan_out, c->plan.bindings.data(), c->plan.bindings.size() * sizeof(pask_binding));
+  c->have_model = true;
+  c->first_done = false;
+  return PASK_OK;
+}
+
+PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, void* stream) {
+  t_err.clear();
+  if (!c) return set_err(PASK_EINVAL, "null ctx");
+  if (!c->have_model) return set_err(PASK_ESTATE, "pask_infer before pask_load_model");
+  int rc;
+  for (size_t i = 0; inputs && i < c->inputs.size(); ++i)
+    if (inputs[i] && (rc = rebind(c, c->inputs[i], inputs[i]))) return rc;
+  for (size_t i = 0; outputs && i < c->outputs.size(); ++i)
+    if (outputs[i] && (rc = rebind(c, c->outputs[i], outputs[i]))) return rc;
+  const Driver* d = c->d;
+  CUstream s = static_cast<CUstream>(stream);
+  CUlaunchAttribute attr[1];
+  attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+  attr[0].value.programmaticStreamSerializationAllowed = 1;
+  for (size_t i = 0; i < c->launches.size(); ++i) {
+    Launch& L = c->launches[i];
+    if ((rc = wait_kernel(c, L.kernel))) return rc;
+    if (i == 0) d->cuEventRecord(c->ev0, s);
+    if (c->cfg.instrument) d->cuEventRecord(c->node_ev[2 * i], s);
+    CUlaunchConfig cfg{};
+    cfg.gridDimX = L.grid[0];
+    cfg.gridDimY = L.grid[1];
+    cfg.gridDimZ = L.grid[2];
+    cfg.blockDimX = L.block[0];
+    cfg.blockDimY = L.block[1];
+    cfg.blockDimZ = L.block[2];
+    cfg.sharedMemBytes = L.smem;
+    cfg.hStream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = (c->cfg.pdl && !c->cfg.instrument && i > 0) ? 1 : 0;
+    void* args[1] = {L.params.get()};
+    const uint64_t t0 = now_ns();
+    CUresult r = d->cuLaunchKernelEx(&cfg, c->fn[L.kernel], args, nullptr);
+    c->st.issue_ns += now_ns() - t0;
+    if (r != CUDA_SUCCESS)
+      return set_err(PASK_ECUDA, cu_err(d, r, ("launch of node " + std::to_string(i) + " (" +
+                                               catalog(L.kernel).name + ")").c_str()));
+    if (c->cfg.instrument) d->cuEventRecord(c->node_ev[2 * i + 1], s);
+    c->st.launches++;
+  }
+  d->cuEventRecord(c->ev1, s);
+  c->st.infer_count++;
+  c->pending = true;
+  return PASK_OK;
+}
+
+PASK_API int pask_sync(pask_ctx* c) {
+  t_err.clear();
+  if (!c) return set_err(PASK_EINVAL, "null ctx");
+  if (!c->pending) return PASK_OK;
+  const Driver* d = c->d;
+  CUresult r = d->cuEventSynchronize(c->ev1);
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuEventSynchronize"));
+  const uint64_t t1 = now_ns();
+  if (!c->first_done) {
+    c->st.cold_wall_ns = t1 - c->t_entry;
+    c->first_done = true;
+  }
+  float ms = 0.f;
+  if (d->cuEventElapsedTime(&ms, c->ev0, c->ev1) == CUDA_SUCCESS)
+    c->st.gpu_span_ns = static_cast<uint64_t>(ms * 1e6);
+  if (c->cfg.instrument) {
+    uint64_t busy = 0;
+    for (size_t i = 0; i + 1 < c->node_ev.size(); i += 2) {
+      float e = 0.f;
+      if (d->cuEventElapsedTime(&e, c->node_ev[i], c->node_ev[i + 1]) == CUDA_SUCCESS)
+        busy += static_cast<uint64_t>(e * 1e6);
+    }
+    c->st.gpu_busy_ns = busy;
+  }
+  c->pending = false;
+  return PASK_OK;
+}
+
+PASK_API int pask_infer_host(pask_ctx* c, const void* const* host_inputs, void* const* host_outputs,
+                             void* stream) {
+  t_err.clear();
+  if (!c) return set_err(PASK_EINVAL, "null ctx");
+  if (!c->have_model) return set_err(PASK_ESTATE, "pask_infer_host before pask_load_model");
+  const Driver* d = c->d;
+  CUstream s = static_cast<CUstream>(stream);
+  for (size_t i = 0; host_inputs && i < c->inputs.size(); ++i) {
+    const pask_tensor& t = c->tensors[c->inputs[i]];
+    CUresult r = d->cuMemcpyHtoDAsync(reinterpret_cast<CUdeviceptr>(t.dptr), host_inputs[i], tensor_bytes(t), s);
+    if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuMemcpyHtoDAsync"));
+  }
+  int rc = pask_infer(c, nullptr, nullptr, stream);
+  if (rc) return rc;
+  for (size_t i = 0; host_outputs && i < c->outputs.size(); ++i) {
+    const pask_tensor& t = c->tensors[c->outputs[i]];
+    CUresult r = d->cuMemcpyDtoHAsync(host_outputs[i], reinterpret_cast<CUdeviceptr>(t.dptr), tensor_bytes(t), s);
+    if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuMemcpyDtoHAsync"));
+  }
+  CUresult r = d->cuStreamSynchronize(s);
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuStreamSynchronize"));
+  return pask_sync(c);
+}
+
+PASK_API int pask_stats(const pask_ctx* c, pask_stats_t* out) {
+  t_err.clear();
+  if (!c || !out) return set_err(PASK_EINVAL, "null ctx or out");
+  *out = c->st;
+  out->kernels_loaded = c->kernels_loaded.load();
+  out->code_objects_loaded = c->code_objects.load();
+  out->code_bytes_loaded = c->code_bytes.load();
+  out->load_ns = c->load_ns.load();
+  return PASK_OK;
+}
+
+PASK_API int pask_kernel_is_loaded(const pask_ctx* c, int32_t k, int32_t* state) {
+  t_err.clear();
+  if (!c || !state || k < 0 || k >= PASK_NUM_KERNELS) return set_err(PASK_EINVAL, "bad argument");
+  *state = 0;
+  if (c->ready[k].load(std::memory_order_acquire) != 1 || !c->fn[k]) return PASK_OK;
+  CUfunctionLoadingState ls;
+  CUresult r = c->d->cuFuncIsLoaded(&ls, c->fn[k]);
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(c->d, r, "cuFuncIsLoaded"));
+  *state = (ls == CU_FUNCTION_LOADING_STATE_LOADED) ? 1 : 0;
+  return PASK_OK;
+}
+
+PASK_API int pask_destroy(pask_ctx* c) {
+  t_err.clear();
+  if (!c) return PASK_OK;
+  {
+    std::lock_guard<std::mutex> lk(c->mu);
+    c->stop = true;
+    c->cv.notify_one();
+  }
+  if (c->loader.joinable()) c->loader.join();
+  const Driver* d = c->d;
+  if (c->pending) d->cuEventSynchronize(c->ev1);
+  for (auto e : c->node_ev)
+    if (e) d->cuEventDestroy(e);
+  if (c->ev0) d->cuEventDestroy(c->ev0);
+  if (c->ev1) d->cuEventDestroy(c->ev1);
+  if (c->lib) d->cuLibraryUnload(c->lib);
+  delete c;
+  return PASK_OK;
+}

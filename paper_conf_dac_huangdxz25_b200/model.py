@@ -1,0 +1,240 @@
+"""Lower a model spec (the lowered layer sequence PASK receives, PAPER.md:91
+Fig. 5) into a pask_graph over caller-owned device memory.
+
+PyTorch is used only to allocate device memory and move bytes (weights,
+inputs); every operator runs in libpask.so.  Device layouts: images NHWC bf16
+(the fp32 NCHW input goes through the layout kernel, C padded to 8), matrices
+row-major bf16, biases / LayerNorm vectors fp32, conv weights KRSC (dense) or
+RSC (depthwise), linear weights [N][K].
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+import torch
+
+from . import pask as P
+
+_ACT = P.ACT
+
+
+class DeviceModel:
+    def __init__(self, spec, device="cuda", solutions=None, alloc=True):
+        """spec: a workloads.models spec.  solutions: {layer index: kernel id}
+        overriding the library's static choice s* for that layer.
+        alloc=False builds the graph with null device pointers (host-only
+        planning / workspace sizing, no GPU needed)."""
+        self.spec = spec
+        self.device = device
+        self.alloc = alloc
+        self.solutions = solutions or {}
+        self.t = {}        # name -> torch tensor (device)
+        self.index = {}    # name -> pask tensor index
+        self.dims = {}     # name -> (n, h, w, c) device dims
+        self.kind = {}     # name -> "image" | "matrix" | "heads"
+        self._tensors = []
+        self._nodes = []
+        self._keep = []
+        self._build()
+
+    # ------------------------------------------------------------ helpers
+    def _dev(self, arr, dtype):
+        if not self.alloc:
+            self._keep.append(arr)
+            return None
+        t = torch.from_numpy(np.ascontiguousarray(arr)).to(dtype).to(self.device)
+        self._keep.append(t)
+        return t
+
+    _FAKE = 1 << 20   # placeholder address for host-only graphs (never dereferenced)
+
+    def _ptr(self, t):
+        if not self.alloc:
+            return self._FAKE
+        return None if t is None else t.data_ptr()
+
+    def _new(self, name, shape, dtype, layout, dims, kind):
+        if self.alloc:
+            t = torch.empty(shape, dtype=dtype, device=self.device)
+            ptr = t.data_ptr()
+        else:
+            t, ptr = None, self._FAKE
+        self.t[name] = t
+        self.dims[name] = dims
+        self.kind[name] = kind
+        self.index[name] = len(self._tensors)
+        pd = P.F32 if dtype == torch.float32 else P.BF16
+        self._tensors.append(P.Tensor(pd, layout, *dims, ptr))
+
+    def _node(self, **kw):
+        nd = P.Node()
+        nd.in1 = nd.res = -1
+        nd.solution = -1
+        for k, v in kw.items():
+            if k in ("stride", "pad", "dil"):
+                getattr(nd, k)[0], getattr(nd, k)[1] = v
+            else:
+                setattr(nd, k, v)
+        self._nodes.append(nd)
+        return nd
+
+    # ------------------------------------------------------------ lowering
+    def _build(self):
+        spec = self.spec
+        for name, shape, dtype in spec["inputs"]:
+            if dtype == "f32":
+                n, c, h, w = shape
+                self._new(name, (n, c, h, w), torch.float32, P.NCHW, (n, h, w, c), "image")
+            else:
+                s, hdim = shape
+                self._new(name, (s, hdim), torch.bfloat16, P.ROWMAJOR, (1, 1, s, hdim), "matrix")
+        for li, L in enumerate(spec["layers"]):
+            op = L["op"]
+            x = L["inputs"][0]
+            xn, xh, xw, xc = self.dims[x]
+            out = L["out"]
+            sol = self.solutions.get(li, -1)
+            if op == "layout":
+                cp = L["c_pad"]
+                self._new(out, (xn, xh, xw, cp), torch.bfloat16, P.NHWC, (xn, xh, xw, cp), "image")
+                self._node(op=P.OP_LAYOUT, in0=self.index[x], out=self.index[out], solution=sol)
+            elif op == "conv":
+                w = L["w"]
+                k, cg, r, s = w.shape
+                groups = L["groups"]
+                _, _, p, q = spec["tensors"][out]
+                if groups == 1:
+                    wd = np.zeros((k, r, s, xc), np.float32)        # KRSC, C padded
+                    wd[..., :cg] = w.transpose(0, 2, 3, 1)
+                else:
+                    wd = w[:, 0].transpose(1, 2, 0)                   # RSC
+                wt = self._dev(wd, torch.bfloat16)
+                bt = self._dev(L["b"], torch.float32) if L["b"] is not None else None
+                bptr = self._ptr(bt) if L["b"] is not None else None
+                self._new(out, (xn, p, q, k), torch.bfloat16, P.NHWC, (xn, p, q, k), "image")
+                self._node(op=P.OP_CONV2D, in0=self.index[x], out=self.index[out],
+                           res=self.index[L["res"]] if L["res"] else -1,
+                           w=self._ptr(wt), bias=bptr, k=k, r=r, s=s,
+                           stride=L["stride"], pad=L["pad"], dil=L["dil"], groups=groups,
+                           act=_ACT[L["act"]], solution=sol)
+            elif op == "pool":
+                _, _, p, q = spec["tensors"][out]
+                self._new(out, (xn, p, q, xc), torch.bfloat16, P.NHWC, (xn, p, q, xc), "image")
+                self._node(op=P.OP_POOL, in0=self.index[x], out=self.index[out],
+                           r=L["kernel"][0], s=L["kernel"][1], stride=L["stride"], pad=L["pad"],
+                           pool_mode=0 if L["mode"] == "max" else 1,
+                           count_include_pad=1 if L["count_include_pad"] else 0,
+                           global_pool=1 if L["global_"] else 0, solution=sol)
+            elif op == "linear":
+                w = L["w"]
+                nout, kin = w.shape
+                if self.kind[x] == "image":
+                    # logical NCHW flatten of an NHWC device tensor: permute W's columns
+                    lc = spec["tensors"][x][1]
+                    wd = w.reshape(nout, lc, xh, xw).transpose(0, 2, 3, 1)
+                    if xc != lc:
+                        wd = np.concatenate([wd, np.zeros((nout, xh, xw, xc - lc), np.float32)], -1)
+                    wd = wd.reshape(nout, -1)
+                    m, kk = xn, xh * xw * xc
+                else:
+                    wd = w
+                    m, kk = xw, xc
+                if L["rows"] is not None:
+                    m = L["rows"]
+                wt = self._dev(wd, torch.bfloat16)
+                bt = self._dev(L["b"], torch.float32) if L["b"] is not None else None
+                bptr = self._ptr(bt) if L["b"] is not None else None
+                self._new(out, (m, nout), torch.bfloat16, P.ROWMAJOR, (1, 1, m, nout), "matrix")
+                self._node(op=P.OP_GEMM, in0=self.index[x], out=self.index[out],
+                           res=self.index[L["res"]] if L["res"] else -1,
+                           w=self._ptr(wt), bias=bptr, m=m, n=nout, kk=kk, batch=1,
+                           trans_b=1, lda=kk, ldb=kk, ldc=nout, act=_ACT[L["act"]], solution=sol)
+            elif op in ("softmax", "layernorm"):
+                shape = tuple(self.t[x].shape) if self.alloc else None
+                dims = self.dims[x]
+                if self.kind[x] == "heads":
+                    shp = (dims[0], dims[2], dims[3])
+                elif self.kind[x] == "matrix":
+                    shp = (dims[2], dims[3])
+                else:
+                    shp = shape
+                self._new(out, shp, torch.bfloat16, P.ROWMAJOR, dims, self.kind[x])
+                if op == "softmax":
+                    self._node(op=P.OP_SOFTMAX, in0=self.index[x], out=self.index[out],
+                               scale=L["scale"], solution=sol)
+                else:
+                    g = self._dev(L["gamma"], torch.float32)
+                    b = self._dev(L["beta"], torch.float32)
+                    self._node(op=P.OP_LAYERNORM, in0=self.index[x], out=self.index[out],
+                               gamma=self._ptr(g), beta=self._ptr(b), eps=L["eps"], solution=sol)
+            elif op == "qk":
+                heads, dh = L["heads"], L["head_dim"]
+                s_, three_h = xw, xc
+                hid = three_h // 3
+                self._new(out, (heads, s_, s_), torch.bfloat16, P.ROWMAJOR, (heads, 1, s_, s_),
+                          "heads")
+                self._node(op=P.OP_GEMM, in0=self.index[x], in1=self.index[x],
+                           out=self.index[out], m=s_, n=s_, kk=dh, batch=heads, trans_b=1,
+                           lda=three_h, ldb=three_h, ldc=s_, off_a=0, off_b=hid, off_c=0,
+                           stride_a=dh, stride_b=dh, stride_c=s_ * s_, act=0, solution=sol)
+            elif op == "pv":
+                heads, dh = L["heads"], L["head_dim"]
+                qkv = L["inputs"][1]
+                s_, three_h = self.dims[qkv][2], self.dims[qkv][3]
+                hid = three_h // 3
+                self._new(out, (s_, hid), torch.bfloat16, P.ROWMAJOR, (1, 1, s_, hid), "matrix")
+                self._node(op=P.OP_GEMM, in0=self.index[x], in1=self.index[qkv],
+                           out=self.index[out], m=s_, n=dh, kk=s_, batch=heads, trans_b=0,
+                           lda=s_, ldb=three_h, ldc=hid, off_a=0, off_b=2 * hid, off_c=0,
+                           stride_a=s_ * s_, stride_b=dh, stride_c=dh, act=0, solution=sol)
+            else:
+                raise ValueError(op)
+        self.inputs = [self.index[n] for n, _, _ in spec["inputs"]]
+        self.outputs = [self.index[n] for n in spec["outputs"]]
+        self._make_graph(None, 0)
+        self.ws_bytes = P.workspace_bytes(self.graph)
+        if self.alloc and self.ws_bytes:
+            self.ws = torch.zeros(self.ws_bytes, dtype=torch.uint8, device=self.device)
+            self._make_graph(self.ws.data_ptr(), self.ws_bytes)
+        else:
+            self.ws = None
+
+    def _make_graph(self, ws, ws_bytes):
+        self._t_arr = (P.Tensor * len(self._tensors))(*self._tensors)
+        self._n_arr = (P.Node * len(self._nodes))(*self._nodes)
+        self._i_arr = (C.c_int32 * len(self.inputs))(*self.inputs)
+        self._o_arr = (C.c_int32 * len(self.outputs))(*self.outputs)
+        self.graph = P.Graph(len(self._tensors), self._t_arr, len(self._nodes), self._n_arr,
+                             len(self.inputs), self._i_arr, len(self.outputs), self._o_arr,
+                             ws, ws_bytes)
+
+    # ------------------------------------------------------------ data movement
+    def set_input(self, x):
+        (name, _, dtype), = self.spec["inputs"]
+        src = torch.from_numpy(np.ascontiguousarray(x))
+        self.t[name].copy_(src.to(self.t[name].dtype))
+
+    def read(self, name):
+        """Device tensor -> float64 numpy in logical layout (NCHW images without
+        channel padding, [rows, cols] matrices, [heads, S, S] scores)."""
+        t = self.t[name].float().cpu().numpy().astype(np.float64)
+        if self.kind[name] == "image" and t.ndim == 4 and self._tensors[self.index[name]].layout \
+                != P.NCHW:
+            lc = self.spec["tensors"][name][1]
+            return t.transpose(0, 3, 1, 2)[:, :lc]
+        return t
+
+    def read_raw(self, name):
+        return self.t[name].float().cpu().numpy().astype(np.float64)
+
+    def write(self, name, arr_logical):
+        """Write a logical-layout array into a device tensor (teacher forcing)."""
+        t = self.t[name]
+        a = np.asarray(arr_logical, dtype=np.float32)
+        if self.kind[name] == "image" and t.ndim == 4 and self._tensors[self.index[name]].layout \
+                != P.NCHW:
+            full = np.zeros(tuple(t.shape), np.float32)
+            full[..., :a.shape[1]] = a.transpose(0, 2, 3, 1)
+            a = full
+        t.copy_(torch.from_numpy(a.reshape(tuple(t.shape))).to(t.dtype))

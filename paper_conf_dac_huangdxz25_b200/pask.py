@@ -1,0 +1,203 @@
+"""Thin ctypes binding of libpask.so (include/pask.h): argument marshalling only.
+
+Every step of the hot path (planning, loading, issuing, all kernels) runs in
+libpask.so; this module only mirrors the C structs and forwards calls.  It
+fails loudly when the library is missing -- there is no Python or CPU fallback.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libpask.so")
+
+# ---------------------------------------------------------------- enums (pask.h)
+OK, EINVAL, EUNSUPPORTED, ECUDA, ENOMEM, ESTATE = 0, -1, -2, -3, -4, -5
+BF16, F32 = 0, 1
+NCHW, NHWC, ROWMAJOR = 0, 1, 2
+OP_LAYOUT, OP_CONV2D, OP_GEMM, OP_POOL, OP_SOFTMAX, OP_LAYERNORM = range(6)
+ACT = {"none": 0, "relu": 1, "relu6": 2, "gelu": 3, "tanh": 4}
+K_LAYOUT, K_CONV_IGEMM, K_CONV_1X1, K_CONV_DW, K_POOL, K_POOL_GAVG, K_GEMM, K_SOFTMAX, \
+    K_LAYERNORM = range(9)
+NUM_KERNELS = 9
+HOW = {0: "direct", 1: "reused", 2: "loaded"}
+
+
+class Tensor(C.Structure):
+    _fields_ = [("dtype", C.c_int32), ("layout", C.c_int32), ("n", C.c_int32),
+                ("h", C.c_int32), ("w", C.c_int32), ("c", C.c_int32), ("dptr", C.c_void_p)]
+
+
+class Node(C.Structure):
+    _fields_ = [("op", C.c_int32), ("in0", C.c_int32), ("in1", C.c_int32), ("res", C.c_int32),
+                ("out", C.c_int32), ("w", C.c_void_p), ("bias", C.c_void_p),
+                ("gamma", C.c_void_p), ("beta", C.c_void_p), ("k", C.c_int32),
+                ("r", C.c_int32), ("s", C.c_int32), ("stride", C.c_int32 * 2),
+                ("pad", C.c_int32 * 2), ("dil", C.c_int32 * 2), ("groups", C.c_int32),
+                ("m", C.c_int32), ("n", C.c_int32), ("kk", C.c_int32), ("batch", C.c_int32),
+                ("trans_b", C.c_int32), ("lda", C.c_int64), ("ldb", C.c_int64),
+                ("ldc", C.c_int64), ("off_a", C.c_int64), ("off_b", C.c_int64),
+                ("off_c", C.c_int64), ("stride_a", C.c_int64), ("stride_b", C.c_int64),
+                ("stride_c", C.c_int64), ("pool_mode", C.c_int32),
+                ("count_include_pad", C.c_int32), ("global_pool", C.c_int32),
+                ("eps", C.c_float), ("scale", C.c_float), ("act", C.c_int32),
+                ("solution", C.c_int32)]
+
+
+class Graph(C.Structure):
+    _fields_ = [("n_tensors", C.c_int32), ("tensors", C.POINTER(Tensor)),
+                ("n_nodes", C.c_int32), ("nodes", C.POINTER(Node)),
+                ("n_inputs", C.c_int32), ("inputs", C.POINTER(C.c_int32)),
+                ("n_outputs", C.c_int32), ("outputs", C.POINTER(C.c_int32)),
+                ("workspace", C.c_void_p), ("workspace_bytes", C.c_uint64)]
+
+
+class Config(C.Structure):
+    _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
+                ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32)]
+
+
+class Binding(C.Structure):
+    _fields_ = [("node", C.c_int32), ("desired_kernel", C.c_int32), ("bound_kernel", C.c_int32),
+                ("how", C.c_int32), ("lookups", C.c_int32)]
+
+
+class Stats(C.Structure):
+    _fields_ = [("n_nodes", C.c_int32), ("kernels_loaded", C.c_int32),
+                ("code_objects_loaded", C.c_int32), ("queries", C.c_int32), ("hits", C.c_int32),
+                ("lookups", C.c_int32), ("code_bytes_loaded", C.c_uint64), ("plan_ns", C.c_uint64),
+                ("load_ns", C.c_uint64), ("load_exposed_ns", C.c_uint64), ("issue_ns", C.c_uint64),
+                ("encode_ns", C.c_uint64), ("gpu_span_ns", C.c_uint64), ("gpu_busy_ns", C.c_uint64),
+                ("cold_wall_ns", C.c_uint64), ("infer_count", C.c_uint64), ("launches", C.c_uint64)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "pask_load_model",
+           "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
+           "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name"]
+
+_lib = None
+
+
+def lib():
+    """Load libpask.so (build it first with paper_conf_dac_huangdxz25_b200.build)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} is missing: run `python -m paper_conf_dac_huangdxz25_b200."
+                           "build` (there is no fallback path)")
+    L = C.CDLL(LIB_PATH)
+    P = C.c_void_p
+    sig = {
+        "pask_version": (C.c_int, []),
+        "pask_create": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(Config)]),
+        "pask_plan": (C.c_int, [C.POINTER(Graph), C.POINTER(Config), C.POINTER(Binding),
+                                C.POINTER(Stats)]),
+        "pask_workspace_bytes": (C.c_int, [C.POINTER(Graph), C.POINTER(C.c_uint64)]),
+        "pask_load_model": (C.c_int, [P, C.POINTER(Graph), C.POINTER(Binding)]),
+        "pask_infer": (C.c_int, [P, C.POINTER(P), C.POINTER(P), P]),
+        "pask_infer_host": (C.c_int, [P, C.POINTER(P), C.POINTER(P), P]),
+        "pask_sync": (C.c_int, [P]),
+        "pask_stats": (C.c_int, [P, C.POINTER(Stats)]),
+        "pask_kernel_is_loaded": (C.c_int, [P, C.c_int32, C.POINTER(C.c_int32)]),
+        "pask_destroy": (C.c_int, [P]),
+        "pask_last_error": (C.c_char_p, []),
+        "pask_num_kernels": (C.c_int32, []),
+        "pask_kernel_name": (C.c_char_p, [C.c_int32]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+class PaskError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"pask error {code}: {msg}")
+        self.code = code
+
+
+def _check(rc):
+    if rc != OK:
+        raise PaskError(rc, lib().pask_last_error().decode())
+    return rc
+
+
+def kernel_name(k):
+    return lib().pask_kernel_name(k).decode()
+
+
+def config(reuse=1, search=0, milestone=0, proactive=1, pdl=1, instrument=0):
+    return Config(reuse, search, milestone, proactive, pdl, instrument)
+
+
+def plan(graph: Graph, cfg: Config | None = None):
+    """Host-only Algorithm 1 plan: (bindings list of tuples, stats dict)."""
+    n = graph.n_nodes
+    out = (Binding * max(n, 1))()
+    st = Stats()
+    _check(lib().pask_plan(C.byref(graph), C.byref(cfg) if cfg else None, out, C.byref(st)))
+    return [(b.node, b.desired_kernel, b.bound_kernel, b.how, b.lookups) for b in out[:n]], \
+        st.as_dict()
+
+
+def workspace_bytes(graph: Graph) -> int:
+    v = C.c_uint64()
+    _check(lib().pask_workspace_bytes(C.byref(graph), C.byref(v)))
+    return v.value
+
+
+class Context:
+    """One pask_ctx (not thread-safe; one per thread)."""
+
+    def __init__(self, device=0, cfg: Config | None = None):
+        self.h = C.c_void_p()
+        _check(lib().pask_create(C.byref(self.h), device, C.byref(cfg) if cfg else None))
+        self.n_nodes = 0
+
+    def load_model(self, graph: Graph):
+        self.n_nodes = graph.n_nodes
+        out = (Binding * max(graph.n_nodes, 1))()
+        _check(lib().pask_load_model(self.h, C.byref(graph), out))
+        return [(b.node, b.desired_kernel, b.bound_kernel, b.how, b.lookups)
+                for b in out[:graph.n_nodes]]
+
+    def infer(self, stream=0, inputs=None, outputs=None):
+        ip = (C.c_void_p * len(inputs))(*inputs) if inputs else None
+        op = (C.c_void_p * len(outputs))(*outputs) if outputs else None
+        _check(lib().pask_infer(self.h, ip, op, C.c_void_p(stream)))
+
+    def infer_host(self, host_inputs, host_outputs, stream=0):
+        ip = (C.c_void_p * len(host_inputs))(*host_inputs)
+        op = (C.c_void_p * len(host_outputs))(*host_outputs)
+        _check(lib().pask_infer_host(self.h, ip, op, C.c_void_p(stream)))
+
+    def sync(self):
+        _check(lib().pask_sync(self.h))
+
+    def stats(self):
+        st = Stats()
+        _check(lib().pask_stats(self.h, C.byref(st)))
+        return st.as_dict()
+
+    def kernel_is_loaded(self, k):
+        v = C.c_int32()
+        _check(lib().pask_kernel_is_loaded(self.h, k, C.byref(v)))
+        return bool(v.value)
+
+    def close(self):
+        if self.h:
+            _check(lib().pask_destroy(self.h))
+            self.h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,50 @@
+"""T3/T5 on the GPU: every layer of every config, teacher-forced vs the oracle,
+through the C ABI (pask_load_model -> pask_infer), plus plan / loaded-kernel
+bit-exactness against the plan oracle and cuFuncIsLoaded."""
+import numpy as np
+import pytest
+
+from oracle import plan as OP
+from paper_conf_dac_huangdxz25_b200 import pask as P
+from workloads import build_model
+
+from .gpu_harness import TOL, run_model, teacher_forced_errors
+
+pytestmark = pytest.mark.gpu
+
+MODELS = ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"]
+
+
+@pytest.mark.parametrize("name", MODELS)
+def test_model_layers_teacher_forced(name):
+    spec, x = build_model(name)
+    dm, ctx, plan = run_model(spec, x)
+    errs = teacher_forced_errors(dm, spec, x)
+    bad = [(i, op, e) for i, op, e in errs if not e <= TOL]
+    assert not bad, f"layers over tolerance: {bad[:10]}"
+    # integer bookkeeping: plan == plan oracle, loaded set == cuFuncIsLoaded
+    o = OP.execution_plan(OP.problems_from_spec(spec))
+    assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
+    st = ctx.stats()
+    assert st["kernels_loaded"] == len(o["loaded"])
+    assert st["code_objects_loaded"] == 1
+    loaded = {k for k in range(P.NUM_KERNELS) if ctx.kernel_is_loaded(k)}
+    assert loaded == set(o["loaded"])
+    assert len(loaded) <= 8
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", MODELS)
+def test_model_hot_repeat_bitwise(name):
+    """A second (hot) inference reproduces the first bit for bit (deterministic
+    split-K; no atomics in any reduction order)."""
+    spec, x = build_model(name)
+    dm, ctx, _ = run_model(spec, x)
+    outs1 = [dm.read_raw(n) for n in spec["outputs"]]
+    import torch
+    ctx.infer(torch.cuda.current_stream().cuda_stream)
+    ctx.sync()
+    outs2 = [dm.read_raw(n) for n in spec["outputs"]]
+    for a, b in zip(outs1, outs2):
+        np.testing.assert_array_equal(a, b)
+    ctx.close()
