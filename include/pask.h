@@ -257,6 +257,16 @@ int pask_stats(const pask_ctx *ctx, pask_stats_t *out);
  * in this context (cuFuncIsLoaded), 0 if not or never requested. */
 int pask_kernel_is_loaded(const pask_ctx *ctx, int32_t kernel_id, int32_t *state);
 
+/* Cold-start timeline of one catalog kernel in this context (host clock, ns
+ * relative to the last pask_load_model entry; 0 when not loaded):
+ *   load_ns     time spent loading it (cuLibraryGetKernel + cuKernelGetFunction
+ *               + cuFuncLoad + attributes; the first load also includes
+ *               cuLibraryLoadData, reported separately in lib_ns),
+ *   ready_ns    when its ready flag was published,
+ *   lib_ns      cuLibraryLoadData time if this kernel's load performed it. */
+int pask_kernel_timeline(const pask_ctx *ctx, int32_t kernel_id, uint64_t *load_ns,
+                         uint64_t *ready_ns, uint64_t *lib_ns);
+
 /* Join the loader thread, unload the library and free host state. */
 int pask_destroy(pask_ctx *ctx);
 

@@ -14,17 +14,20 @@
 //   conv: m = output pixel (n, p, q), n = output channel, k = (r, s, c) in KRSC order,
 //         A[m][k] = X[n, p*sh - ph + r*dh, q*sw - pw + s*dw, c] (0 outside)
 //
-// Structure (192 threads, one 128 x BN output tile per CTA):
-//   warps 0-3 : A_GATHER -> implicit im2col producer (cp.async, 16 B per lane,
-//               SWIZZLE_128B placement); then the epilogue (TMEM -> registers ->
-//               bias / residual / activation -> bf16 NHWC stores, or split-K)
-//   warp 4    : TMA producer (B always; A in A_TMA mode)
+// Structure (192 threads, one 128 x BN output tile per CTA, or per cluster):
+//   warps 0-3 : bias -> smem; A_GATHER: implicit im2col producer (cp.async,
+//               16 B per lane, SWIZZLE_128B placement); then the epilogue
+//   warp 4    : TMA producer (B always, A in A_TMA mode, the residual tile)
 //   warp 5    : TMEM allocator + single-thread tcgen05.mma issuer
-//   smem ring : `stages` x {A 128x64, B BNx64} bf16, full/empty mbarriers
-//   split-K   : deterministic -- every split writes an fp32 partial tile; the
-//               last-arriving CTA (atomic ticket) sums the partials in split
-//               order 0..S-1 and runs the epilogue, so a given (kernel, problem)
-//               is bitwise reproducible (SURVEY.md §7 hard part 8).
+//   smem      : ring of `stages` x {A 128x64, B BNx64} bf16 with full/empty
+//               mbarriers; residual/output staging tile; bias vector
+//   epilogue  : TMEM -> registers -> (+bias, +residual from smem, act) -> bf16
+//               staged in smem -> TMA tensor store (clips the M / N tails)
+//   split-K   : a thread-block cluster of S = 2/4/8 CTAs along z, one K range
+//               each; every CTA parks its fp32 tile in its own smem, then rank
+//               r reduces rows [r*128/S, (r+1)*128/S) over the S peers through
+//               DSMEM in fixed rank order 0..S-1 -- deterministic, so a given
+//               (kernel, problem) is bitwise reproducible (SURVEY.md §7 part 8).
 #pragma once
 #include "pask_params.h"
 #include "ptx.cuh"
@@ -35,91 +38,146 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// Epilogue for 16 consecutive output columns of one row.
-__device__ __forceinline__ void store_row16(const GemmParams& p, int b, int m, int n0,
-                                            float (&v)[16]) {
-  const int64_t base = p.off_c + (int64_t)b * p.stride_c + (int64_t)m * p.ldc + n0;
-  const bool full = (n0 + 16 <= p.N) && ((base & 7) == 0);
-  if (p.bias) {
+// Activation over 16 values: one loop per activation kind (compact SASS).
+__device__ __forceinline__ void act16(float (&v)[16], int act) {
+  if (act == 1) {
 #pragma unroll
-    for (int i = 0; i < 16; ++i)
-      if (n0 + i < p.N) v[i] += __ldg(p.bias + n0 + i);
+    for (int i = 0; i < 16; ++i) v[i] = fmaxf(v[i], 0.f);
+  } else if (act == 2) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = fminf(fmaxf(v[i], 0.f), 6.f);
+  } else if (act == 3) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i], 3);
+  } else if (act == 4) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i], 4);
   }
-  const __nv_bfloat16* res = reinterpret_cast<const __nv_bfloat16*>(p.res);
-  __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
-  if (full) {
-    if (res) {
-      uint4 r0 = *reinterpret_cast<const uint4*>(res + base);
-      uint4 r1 = *reinterpret_cast<const uint4*>(res + base + 8);
+}
+
+// Layout of the residual / output staging tile: column boxes of box_cols
+// (16/32/48/64) columns, each 128 rows x box_cols bf16; 64-wide boxes use the
+// TMA SWIZZLE_128B pattern (16 B chunk c of row r at chunk c ^ (r & 7)).
+__device__ __forceinline__ uint32_t ro_chunk(uint32_t ro, int box_cols, int row, int col) {
+  const int j = col / box_cols;
+  const int cc = (col - j * box_cols) >> 3;
+  const uint32_t base = ro + j * (128 * box_cols * 2) + row * (box_cols * 2);
+  return box_cols == 64 ? base + ((cc ^ (row & 7)) << 4) : base + (cc << 4);
+}
+
+struct EpiCtx {
+  const float* s_bias;  // smem, bn floats (0 outside N)
+  uint32_t ro;          // smem staging tile (c_tma)
+  int box_cols;
+  int m0, n0, b;
+};
+
+// v = act(acc + bias + res) -> bf16 (RNE) for 16 columns of tile row `row`:
+// staged in smem for the TMA store (c_tma) or stored directly (unaligned output).
+__device__ __forceinline__ void epi16(const GemmParams& p, const EpiCtx& e, int row, int cb,
+                                      float (&v)[16]) {
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] += e.s_bias[cb + i];
+  const int m = e.m0 + row, n = e.n0 + cb;
+  const uint32_t a0 = ro_chunk(e.ro, e.box_cols, row, cb);
+  const uint32_t a1 = ro_chunk(e.ro, e.box_cols, row, cb + 8);
+  const bool in = m < p.M && n < p.N;
+  const int nv = min(16, p.N - n);
+  const int64_t base = p.off_c + static_cast<int64_t>(e.b) * p.stride_c + static_cast<int64_t>(m) * p.ldc + n;
+  if (p.res) {
+    float f[16];
+    if (p.c_tma) {
+      uint4 r0, r1;
+      asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r0.x), "=r"(r0.y), "=r"(r0.z), "=r"(r0.w) : "r"(a0));
+      asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r1.x), "=r"(r1.y), "=r"(r1.z), "=r"(r1.w) : "r"(a1));
       float f0[8], f1[8];
       unpack_bf16x8(r0, f0);
       unpack_bf16x8(r1, f1);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        v[i] += f0[i];
-        v[8 + i] += f1[i];
+        f[i] = f0[i];
+        f[8 + i] = f1[i];
       }
-    }
-    float a0[8], a1[8];
+    } else {
+      const __nv_bfloat16* res = reinterpret_cast<const __nv_bfloat16*>(p.res);
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      a0[i] = apply_act(v[i], p.act);
-      a1[i] = apply_act(v[8 + i], p.act);
+      for (int i = 0; i < 16; ++i) f[i] = (in && i < nv) ? __bfloat162float(res[base + i]) : 0.f;
     }
-    *reinterpret_cast<uint4*>(out + base) = pack_bf16x8(a0);
-    *reinterpret_cast<uint4*>(out + base + 8) = pack_bf16x8(a1);
-  } else {
 #pragma unroll
-    for (int i = 0; i < 16; ++i) {
-      if (n0 + i < p.N) {
-        float t = v[i];
-        if (res) t += __bfloat162float(res[base + i]);
-        out[base + i] = __float2bfloat16_rn(apply_act(t, p.act));
-      }
-    }
+    for (int i = 0; i < 16; ++i) v[i] += f[i];
+  }
+  act16(v, p.act);
+  uint32_t pk[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) pk[i] = pack_bf16x2(v[2 * i], v[2 * i + 1]);
+  if (p.c_tma) {
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a0), "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]) : "memory");
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a1), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]) : "memory");
+  } else if (in) {
+    unsigned short* o16 = reinterpret_cast<unsigned short*>(p.out) + base;
+#pragma unroll
+    for (int i = 0; i < 16; ++i)
+      if (i < nv) o16[i] = static_cast<unsigned short>((pk[i >> 1] >> (16 * (i & 1))) & 0xFFFFu);
   }
 }
 
 template <bool kAllowGather>
 __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   extern __shared__ uint8_t smem_raw[];
-  __shared__ uint32_t s_last;
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  const int t = threadIdx.x;
   const int stages = p.stages;
   const int bn = p.bn;
+  const int splits = p.splits;
   constexpr uint32_t kABytes = kBM * kBK * 2;  // 16 KB
   const uint32_t b_bytes = static_cast<uint32_t>(bn) * kBK * 2;
   const uint32_t stage_bytes = kABytes + b_bytes;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + stages * stage_bytes);
+  // ---- smem carve-up (mirrors gemm_tiling() on the host)
+  const uint32_t ring_bytes = stages * stage_bytes;
+  const uint32_t stage32_pitch = (bn + 4) * 4;  // fp32 split-K staging row pitch (bank spread)
+  const uint32_t reg0 = (max(ring_bytes, splits > 1 ? 128u * stage32_pitch : 0u) + 1023u) & ~1023u;
+  const uint32_t ro_bytes = p.c_tma ? ((128u * bn * 2 + 1023u) & ~1023u) : 0u;
+  float* s_bias = reinterpret_cast<float*>(smem + reg0 + ro_bytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + reg0 + ro_bytes + 1024);
+  const uint32_t smem_base = smem_u32(smem);
   const uint32_t full0 = smem_u32(bars);
   const uint32_t empty0 = smem_u32(bars + stages);
   const uint32_t accum_bar = smem_u32(bars + 2 * stages);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * stages + 1);
-  const uint32_t smem_base = smem_u32(smem);
+  const uint32_t res_bar = smem_u32(bars + 2 * stages + 1);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * stages + 2);
+  const uint32_t ro = smem_base + reg0;
 
   const bool gather = kAllowGather && (p.a_mode == A_GATHER);
   const int mt = blockIdx.x, nt = blockIdx.y;
-  const int b = blockIdx.z / p.splits;
-  const int split = blockIdx.z - b * p.splits;
-  const int kb_begin = split * p.kb_per_split;
-  const int kb_end = min(p.num_kb, kb_begin + p.kb_per_split);
-  const int nk = kb_end - kb_begin;  // >= 1 (host guarantees)
+  const int b = blockIdx.z / splits;
+  const int split = blockIdx.z - b * splits;
+  const int kb_begin = static_cast<int>((static_cast<int64_t>(split) * p.num_kb) / splits);
+  const int kb_end = static_cast<int>((static_cast<int64_t>(split + 1) * p.num_kb) / splits);
+  const int nk = kb_end - kb_begin;  // >= 1 (host guarantees num_kb >= splits)
+  const int m0 = mt * kBM, n0 = nt * bn;
+  const int box_cols = bn < 64 ? bn : 64;
+  const int rows_per = p.rows_per;
+  const int r0 = splits > 1 ? static_cast<int>(cluster_ctarank()) * rows_per : 0;
+  const bool res_tma = p.c_tma && p.res != nullptr;
 
   // ---------------- prologue (overlaps the previous kernel under PDL)
-  if (threadIdx.x == 0) {
+  if (t == 0) {
     for (int s = 0; s < stages; ++s) {
       mbar_init(full0 + 8 * s, gather ? 129u : 1u);
       mbar_init(empty0 + 8 * s, 1u);
     }
     mbar_init(accum_bar, 1u);
+    mbar_init(res_bar, 1u);
     fence_barrier_init();
   }
   if (warp == 4 && lane == 0) {
     if (!gather) tma_prefetch_desc(&p.tmap_a);
     tma_prefetch_desc(&p.tmap_b);
+    if (p.c_tma) tma_prefetch_desc(&p.tmap_c);
+    if (res_tma) tma_prefetch_desc(&p.tmap_r);
   }
   if (warp == 5) tmem_alloc(smem_u32(tmem_slot), p.tmem_cols);
   tc_fence_before();
@@ -133,6 +191,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   if (warp == 4) {
     // ================= TMA producer
     if (lane == 0) {
+      if (res_tma) {  // residual rows [r0, r0 + rows_per) of the tile, consumed by the epilogue
+        mbar_arrive_expect_tx(res_bar, static_cast<uint32_t>(rows_per * bn * 2));
+        for (int j = 0; j < bn / box_cols; ++j)
+          tma_load_3d(ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), &p.tmap_r, res_bar,
+                      n0 + j * box_cols, m0 + r0, b);
+      }
       for (int i = 0; i < nk; ++i) {
         const int s = i % stages;
         const uint32_t ph = (i / stages) & 1;
@@ -141,15 +205,16 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const uint32_t sb = sa + kABytes;
         const int kb = kb_begin + i;
         mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
-        if (!gather) tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, mt * kBM, b);
+        if (!gather) tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
         if (p.b_major == 0) {
-          tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, nt * bn, b);
+          tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
         } else {
           for (int j = 0; j < bn / 64; ++j)
-            tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * s, nt * bn + j * 64, kb * kBK, b);
+            tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * s, n0 + j * 64, kb * kBK, b);
         }
       }
     }
+    __syncwarp();
   } else if (warp == 5) {
     // ================= MMA issuer (one thread issues for the whole CTA)
     if (lane == 0) {
@@ -176,8 +241,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
     }
     __syncwarp();
   } else {
-    // ================= warps 0-3
-    const int t = threadIdx.x;  // 0..127
+    // ================= warps 0-3: bias, (gather), epilogue
+    if (t < bn) s_bias[t] = (p.bias != nullptr && n0 + t < p.N) ? __ldg(p.bias + n0 + t) : 0.f;
     if (kAllowGather && gather) {
       // implicit im2col: lane t owns 16 B chunk j = t % 8 of rows rg + 16 * ri
       const int j = t & 7;
@@ -188,7 +253,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       const int pq = p.P * p.Q;
 #pragma unroll
       for (int ri = 0; ri < 8; ++ri) {
-        const int m = mt * kBM + rg + 16 * ri;
+        const int m = m0 + rg + 16 * ri;
         rv[ri] = m < p.M;
         const int mm = rv[ri] ? m : 0;
         const int n = mm / pq;
@@ -243,67 +308,77 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       fence_proxy_async_smem();
       for (int i = max(0, nk - lag); i < nk; ++i) mbar_arrive(full0 + 8 * (i % stages));
     }
-
-    // ---------------- epilogue: TMEM lane == tile row
+    named_bar_sync(1, 128);  // s_bias complete
     mbar_wait(accum_bar, 0);
     tc_fence_after();
-    const int row = warp * 32 + lane;
-    const int m = mt * kBM + row;
-    const uint32_t taddr = tmem_base + (static_cast<uint32_t>(warp * 32) << 16);
-    if (p.splits == 1) {
-      for (int cb = 0; cb < bn; cb += 16) {
-        float v[16];
-        tmem_ld16(taddr + cb, v);
-        const int n0 = nt * bn + cb;
-        if (m < p.M && n0 < p.N) store_row16(p, b, m, n0, v);
-      }
-    } else {
-      const int tile = (b * p.m_tiles + mt) * p.n_tiles + nt;
-      float* part = p.ws_partial + (static_cast<int64_t>(tile * p.splits + split) * kBM + row) * bn;
+  }
+
+  // ---------------- epilogue
+  EpiCtx e{s_bias, ro, box_cols, m0, n0, b};
+  const uint32_t taddr = tmem_base + (static_cast<uint32_t>((warp & 3) * 32) << 16);
+  const int cpr = bn >> 4;  // 16-column chunks per row
+  if (splits > 1) {
+    // park this split's fp32 tile in smem (ring is idle: all MMAs completed)
+    if (warp < 4) {
+      const int row = warp * 32 + lane;
+      const uint32_t dst = smem_base + row * stage32_pitch;
       for (int cb = 0; cb < bn; cb += 16) {
         float v[16];
         tmem_ld16(taddr + cb, v);
 #pragma unroll
         for (int q4 = 0; q4 < 4; ++q4)
-          __stcg(reinterpret_cast<float4*>(part + cb) + q4,
-                 make_float4(v[4 * q4], v[4 * q4 + 1], v[4 * q4 + 2], v[4 * q4 + 3]));
-      }
-      __threadfence();
-      named_bar_sync(1, 128);
-      if (t == 0) {
-        const uint32_t old = atomicAdd(p.ws_counter + tile, 1u);
-        s_last = (old == static_cast<uint32_t>(p.splits - 1)) ? 1u : 0u;
-      }
-      named_bar_sync(1, 128);
-      if (s_last) {
-        __threadfence();
-        const float* base = p.ws_partial + (static_cast<int64_t>(tile * p.splits) * kBM + row) * bn;
-        if (m < p.M) {
-          for (int cb = 0; cb < bn; cb += 16) {
-            const int n0 = nt * bn + cb;
-            if (n0 >= p.N) break;
-            float v[16];
-#pragma unroll
-            for (int i = 0; i < 16; ++i) v[i] = 0.f;
-            for (int sp = 0; sp < p.splits; ++sp) {  // fixed order: deterministic
-              const float4* src = reinterpret_cast<const float4*>(
-                  base + static_cast<int64_t>(sp) * kBM * bn + cb);
-#pragma unroll
-              for (int q4 = 0; q4 < 4; ++q4) {
-                const float4 f = __ldcg(src + q4);
-                v[4 * q4] += f.x;
-                v[4 * q4 + 1] += f.y;
-                v[4 * q4 + 2] += f.z;
-                v[4 * q4 + 3] += f.w;
-              }
-            }
-            store_row16(p, b, m, n0, v);
-          }
-        }
-        if (t == 0) p.ws_counter[tile] = 0u;  // self-reset for the next layer / inference
+          asm volatile("st.shared.v4.f32 [%0], {%1,%2,%3,%4};" ::"r"(dst + (cb + 4 * q4) * 4),
+                       "f"(v[4 * q4]), "f"(v[4 * q4 + 1]), "f"(v[4 * q4 + 2]), "f"(v[4 * q4 + 3])
+                       : "memory");
       }
     }
+    cluster_sync_all();  // every split's partial tile is parked
   }
+  if (warp < 4) {
+    if (res_tma) mbar_wait(res_bar, 0);
+    // items: (row, 16-column chunk).  splits == 1: thread t owns TMEM lane / row t.
+    // splits > 1: the 128 threads stride over this rank's rows_per x cpr items.
+    const int n_items = splits == 1 ? cpr : (rows_per * cpr - t + 127) / 128;
+    for (int k = 0; k < n_items; ++k) {
+      int row, cb;
+      float v[16];
+      if (splits == 1) {
+        row = t;
+        cb = k << 4;
+        tmem_ld16(taddr + cb, v);  // warp-collective
+      } else {
+        const int it = t + 128 * k;
+        row = r0 + it / cpr;
+        cb = (it - (it / cpr) * cpr) << 4;
+        const uint32_t local = smem_base + row * stage32_pitch + cb * 4;
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = 0.f;
+        for (int sp = 0; sp < splits; ++sp) {  // fixed rank order: deterministic
+          const uint32_t ra = mapa_cluster(local, static_cast<uint32_t>(sp));
+#pragma unroll
+          for (int q4 = 0; q4 < 4; ++q4) {
+            const float4 f = ld_dsmem_f4(ra + 16 * q4);
+            v[4 * q4] += f.x;
+            v[4 * q4 + 1] += f.y;
+            v[4 * q4 + 2] += f.z;
+            v[4 * q4 + 3] += f.w;
+          }
+        }
+      }
+      epi16(p, e, row, cb, v);
+    }
+  }
+  if (p.c_tma && warp < 4) {
+    fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
+    named_bar_sync(1, 128);
+    if (t == 0) {
+      for (int j = 0; j < bn / box_cols; ++j)
+        tma_store_3d(&p.tmap_c, ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), n0 + j * box_cols,
+                     m0 + r0, b);
+      tma_store_commit_and_wait_read();
+    }
+  }
+  if (splits > 1) cluster_sync_all();  // peers finished reading this CTA's partial tile
 
   // ---------------- teardown
   tc_fence_before();

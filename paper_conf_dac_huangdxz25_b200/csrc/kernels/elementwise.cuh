@@ -45,16 +45,23 @@ __device__ __forceinline__ void layout_body(const LayoutParams& p) {
 }
 
 // ---------------------------------------------------------------- K7 pool
-// One thread per (output pixel, 8-channel chunk).  Max pads with -inf; avg
-// divides by the window or by the in-range count.
+// Small windows: one thread per (output pixel, 8-channel chunk).  Large windows
+// (per_warp, e.g. a 7x7 global pool): one warp per output chunk, lanes stride
+// over the window taps and combine with a fixed shuffle tree (deterministic).
+// Max pads with -inf; avg divides by the window or by the in-range count.
 __device__ __forceinline__ void pool_body(const PoolParams& p) {
   pdl_wait();
   pdl_launch_dependents();
   const int chunks = p.C >> 3;
   const int64_t total = static_cast<int64_t>(p.n) * p.P * p.Q * chunks;
   const uint4* x = reinterpret_cast<const uint4*>(p.x);
-  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < total;
-       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+  const int lane = threadIdx.x & 31;
+  const int64_t first = p.per_warp ? (blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x) >> 5
+                                   : blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
+  const int64_t step = p.per_warp ? (static_cast<int64_t>(gridDim.x) * blockDim.x) >> 5
+                                  : static_cast<int64_t>(gridDim.x) * blockDim.x;
+  const int taps = p.R * p.S;
+  for (int64_t idx = first; idx < total; idx += step) {
     int64_t t = idx;
     const int ch = static_cast<int>(t % chunks);
     t /= chunks;
@@ -65,32 +72,40 @@ __device__ __forceinline__ void pool_body(const PoolParams& p) {
     float acc[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = p.mode == 0 ? -INFINITY : 0.f;
-    int cnt = 0;
+    float cnt = 0.f;
     const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
-    for (int r = 0; r < p.R; ++r) {
-      const int ih = ih0 + r;
-      if (ih < 0 || ih >= p.H) continue;
-      for (int s = 0; s < p.S; ++s) {
-        const int iw = iw0 + s;
-        if (iw < 0 || iw >= p.W) continue;
-        float f[8];
-        unpack_bf16x8(__ldg(x + ((static_cast<int64_t>(n) * p.H + ih) * p.W + iw) * chunks + ch), f);
-        ++cnt;
-        if (p.mode == 0) {
+    for (int tap = p.per_warp ? lane : 0; tap < taps; tap += p.per_warp ? 32 : 1) {
+      const int r = tap / p.S, s = tap - (tap / p.S) * p.S;
+      const int ih = ih0 + r, iw = iw0 + s;
+      if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;
+      float f[8];
+      unpack_bf16x8(__ldg(x + ((static_cast<int64_t>(n) * p.H + ih) * p.W + iw) * chunks + ch), f);
+      cnt += 1.f;
+      if (p.mode == 0) {
 #pragma unroll
-          for (int i = 0; i < 8; ++i) acc[i] = fmaxf(acc[i], f[i]);
-        } else {
+        for (int i = 0; i < 8; ++i) acc[i] = fmaxf(acc[i], f[i]);
+      } else {
 #pragma unroll
-          for (int i = 0; i < 8; ++i) acc[i] += f[i];
+        for (int i = 0; i < 8; ++i) acc[i] += f[i];
+      }
+    }
+    if (p.per_warp) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float other = __shfl_xor_sync(0xffffffffu, acc[i], o);
+          acc[i] = p.mode == 0 ? fmaxf(acc[i], other) : acc[i] + other;
         }
+        cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
       }
     }
     if (p.mode == 1) {
-      const float div = p.count_include_pad ? static_cast<float>(p.R * p.S) : static_cast<float>(cnt);
+      const float div = p.count_include_pad ? static_cast<float>(taps) : cnt;
 #pragma unroll
       for (int i = 0; i < 8; ++i) acc[i] = acc[i] / div;
     }
-    reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(acc);
+    if (!p.per_warp || lane == 0) reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(acc);
   }
 }
 

@@ -21,6 +21,8 @@ enum AMode : int32_t {
 struct alignas(64) GemmParams {
   CUtensorMap tmap_a;  // A_TMA: 3-D {K, M, batch}, box {64, 128, 1}, SWIZZLE_128B
   CUtensorMap tmap_b;  // K-major: {K, N, batch} box {64, BN, 1}; MN-major: {N, K, batch} box {64, 64, 1}
+  CUtensorMap tmap_c;  // c_tma: output {N, M, batch} (ldc), box {64, rows_per, 1}, SWIZZLE_128B
+  CUtensorMap tmap_r;  // c_tma && res: residual, same geometry as tmap_c with box {64, 128, 1}
   const void* x;       // A_GATHER: NHWC bf16 input
   void* out;           // bf16 output (row i of tile at out + off_c + b*stride_c + i*ldc)
   const void* res;     // bf16 residual, same indexing as out (nullable)
@@ -38,6 +40,8 @@ struct alignas(64) GemmParams {
   int32_t b_major;       // 0 K-major, 1 MN-major
   int32_t act;           // pask_act
   int32_t m_tiles, n_tiles;
+  int32_t c_tma;         // 1: output (and residual) through TMA + smem staging
+  int32_t rows_per;      // rows reduced / stored per cluster rank = 128 / splits
   // implicit-GEMM geometry (A_GATHER): input [n][H][W][C], output pixel m -> (n, p, q)
   int32_t H, W, C, P, Q, R, S;
   int32_t sh, sw, ph, pw, dh, dw;
@@ -58,6 +62,7 @@ struct alignas(16) PoolParams {
   int32_t n, H, W, C, P, Q, R, S, sh, sw, ph, pw;
   int32_t mode;   // 0 max, 1 avg
   int32_t count_include_pad;
+  int32_t per_warp;  // 1: one warp per output chunk, lanes split the window (large windows)
 };
 
 struct alignas(16) DwParams {

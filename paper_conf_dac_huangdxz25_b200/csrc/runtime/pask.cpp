@@ -63,6 +63,7 @@ struct Launch {
   unsigned grid[3] = {1, 1, 1};
   unsigned block[3] = {1, 1, 1};
   unsigned smem = 0;
+  unsigned cluster_z = 1;  // split-K cluster size (thread-block cluster along z)
   std::unique_ptr<AnyParams> params;
 };
 
@@ -94,6 +95,9 @@ struct Ctx {
   std::atomic<int32_t> code_objects{0};
   std::atomic<uint64_t> code_bytes{0};
   std::atomic<int32_t> kernels_loaded{0};
+  uint64_t k_load_ns[PASK_NUM_KERNELS] = {};   // per-kernel cold timeline
+  uint64_t k_ready_at[PASK_NUM_KERNELS] = {};  // absolute steady-clock ns
+  uint64_t k_lib_ns[PASK_NUM_KERNELS] = {};
 
   // ---- model
   bool have_model = false;
@@ -138,6 +142,7 @@ void load_kernel(Ctx* c, int32_t k) {
   if (!c->lib) {
     const size_t bytes = static_cast<size_t>(pask_fatbin_end - pask_fatbin_start);
     r = d->cuLibraryLoadData(&c->lib, pask_fatbin_start, nullptr, nullptr, 0, nullptr, nullptr, 0);
+    c->k_lib_ns[k] = now_ns() - t0;
     if (r == CUDA_SUCCESS) {
       c->code_objects.fetch_add(1);
       c->code_bytes.fetch_add(bytes);
@@ -149,11 +154,16 @@ void load_kernel(Ctx* c, int32_t k) {
   if (r == CUDA_SUCCESS) r = d->cuKernelGetFunction(&f, kern);
   if (r == CUDA_SUCCESS) r = d->cuFuncLoad(f);
   if (r == CUDA_SUCCESS && is_gemm_kernel(k))
-    r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 227 * 1024);
+    r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 210 * 1024);  // >= gemm_tiling max (200 KB ring + barriers + align)
+  if (r == CUDA_SUCCESS && is_gemm_kernel(k))  // one fixed L1/smem split: no per-launch reconfiguration
+    r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100);
   c->fn[k] = f;
   c->kerr[k] = r;
   if (r == CUDA_SUCCESS) c->kernels_loaded.fetch_add(1);
-  c->load_ns.fetch_add(now_ns() - t0);
+  const uint64_t t1 = now_ns();
+  c->k_load_ns[k] = t1 - t0;
+  c->k_ready_at[k] = t1;
+  c->load_ns.fetch_add(t1 - t0);
   c->ready[k].store(r == CUDA_SUCCESS ? 1 : -1, std::memory_order_release);
 }
 
@@ -175,7 +185,8 @@ void loader_main(Ctx* c) {
 
 // ------------------------------------------------------------------ tensor maps
 int encode_3d(Ctx* c, CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1, uint64_t d2,
-              uint64_t s1_bytes, uint64_t s2_bytes, uint32_t b0, uint32_t b1, std::string* err) {
+              uint64_t s1_bytes, uint64_t s2_bytes, uint32_t b0, uint32_t b1, std::string* err,
+              CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   if (d2 <= 1) s2_bytes = s1_bytes * d1;
   cuuint64_t dims[3] = {d0, d1, std::max<uint64_t>(d2, 1)};
   cuuint64_t strides[2] = {s1_bytes, s2_bytes};
@@ -183,7 +194,7 @@ int encode_3d(Ctx* c, CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1
   cuuint32_t es[3] = {1, 1, 1};
   CUresult r = c->d->cuTensorMapEncodeTiled(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims,
                                             strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                            swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     *err = cu_err(c->d, r, "cuTensorMapEncodeTiled");
@@ -225,6 +236,7 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
   L.block[1] = L.block[2] = 1;
   L.grid[1] = L.grid[2] = 1;
   L.smem = 0;
+  L.cluster_z = 1;
   switch (L.kernel) {
     case PASK_K_LAYOUT: {
       LayoutParams& q = L.params->l;
@@ -255,7 +267,9 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
         L.grid[0] = static_cast<unsigned>((p.c / 8 + 31) / 32);
         L.grid[1] = static_cast<unsigned>(p.n);
       } else {
-        L.grid[0] = grid_1d(static_cast<int64_t>(p.n) * p.p * p.q * (p.c / 8), 256);
+        const int64_t outs = static_cast<int64_t>(p.n) * p.p * p.q * (p.c / 8);
+        q.per_warp = (p.r * p.s > 16) ? 1 : 0;
+        L.grid[0] = grid_1d(q.per_warp ? outs * 32 : outs, 256);
       }
       return PASK_OK;
     }
@@ -273,27 +287,42 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
       GemmParams& q = L.params->g;
       int32_t M, N, K, batch, b_major;
       contraction_shape(p, nd, &M, &N, &K, &batch, &b_major);
-      const GemmTiling t = gemm_tiling(M, N, K, batch, b_major);
+      const int64_t ldc = p.op == OC_CONV ? p.k : nd.ldc;
+      const int64_t off_c = p.op == OC_CONV ? 0 : nd.off_c;
+      const int64_t stride_c = p.op == OC_CONV ? 0 : nd.stride_c;
+      auto al16 = [](const void* ptr) { return (reinterpret_cast<uintptr_t>(ptr) & 15) == 0; };
+      // staged TMA epilogue needs 16-byte row pitch / offsets (not e.g. the N = 10 FC)
+      const int32_t c_tma = (ldc % 8 == 0) && (off_c % 8 == 0) && (batch == 1 || stride_c % 8 == 0) &&
+                            al16(y.dptr) && (!res || al16(res));
+      const GemmTiling t = gemm_tiling(M, N, K, batch, b_major, c_tma);
       q.M = M; q.N = N; q.K = K; q.batch = batch;
-      q.num_kb = t.num_kb; q.kb_per_split = t.kb_per_split; q.splits = t.splits;
+      q.num_kb = t.num_kb; q.kb_per_split = (t.num_kb + t.splits - 1) / t.splits; q.splits = t.splits;
+      q.rows_per = t.rows_per; q.c_tma = c_tma;
       q.bn = t.bn; q.stages = t.stages; q.b_major = b_major; q.act = nd.act;
       q.m_tiles = t.m_tiles; q.n_tiles = t.n_tiles;
       q.idesc = make_idesc(t.bn, b_major);
       q.tmem_cols = t.tmem_cols;
       q.smem_bytes = t.smem_bytes;
       q.out = y.dptr; q.res = res; q.bias = nd.bias;
-      const uint64_t cnt_region = (t.ws_counter_bytes + 255) / 256 * 256;
-      if (t.splits > 1) {
-        if (!c->ws || c->ws_bytes < cnt_region + t.ws_partial_bytes) {
-          *err = "node " + std::to_string(i) + ": workspace too small (see pask_workspace_bytes)";
-          return PASK_ENOMEM;
-        }
-        q.ws_counter = static_cast<uint32_t*>(c->ws);
-        q.ws_partial = reinterpret_cast<float*>(static_cast<char*>(c->ws) + cnt_region);
-      }
+      q.ldc = ldc; q.off_c = off_c; q.stride_c = stride_c;
       int rc;
+      if (c_tma) {
+        const uint32_t box_cols = t.bn < 64 ? static_cast<uint32_t>(t.bn) : 64u;
+        const CUtensorMapSwizzle swz = box_cols == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE;
+        const char* cbase = static_cast<const char*>(y.dptr) + off_c * 2;
+        rc = encode_3d(c, &q.tmap_c, cbase, static_cast<uint64_t>(N), static_cast<uint64_t>(M),
+                       static_cast<uint64_t>(batch), static_cast<uint64_t>(ldc) * 2,
+                       static_cast<uint64_t>(stride_c) * 2, box_cols, static_cast<uint32_t>(t.rows_per), err, swz);
+        if (rc) return rc;
+        if (res) {
+          const char* rbase = static_cast<const char*>(res) + off_c * 2;
+          rc = encode_3d(c, &q.tmap_r, rbase, static_cast<uint64_t>(N), static_cast<uint64_t>(M),
+                         static_cast<uint64_t>(batch), static_cast<uint64_t>(ldc) * 2,
+                         static_cast<uint64_t>(stride_c) * 2, box_cols, static_cast<uint32_t>(t.rows_per), err, swz);
+          if (rc) return rc;
+        }
+      }
       if (p.op == OC_CONV) {
-        q.ldc = p.k; q.off_c = 0; q.stride_c = 0;
         const bool plain = (p.r == 1 && p.s == 1 && p.stride_h == 1 && p.stride_w == 1 && p.pad_h == 0 &&
                             p.pad_w == 0);
         q.a_mode = (L.kernel == PASK_K_CONV_1X1 || plain) ? A_TMA : A_GATHER;
@@ -310,7 +339,6 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
                        static_cast<uint64_t>(K) * 2, 0, 64, static_cast<uint32_t>(t.bn), err);
         if (rc) return rc;
       } else {
-        q.ldc = nd.ldc; q.off_c = nd.off_c; q.stride_c = nd.stride_c;
         q.a_mode = A_TMA;
         const char* abase = static_cast<const char*>(x.dptr) + nd.off_a * 2;
         rc = encode_3d(c, &q.tmap_a, abase, static_cast<uint64_t>(K), static_cast<uint64_t>(M),
@@ -333,6 +361,7 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
       L.grid[0] = static_cast<unsigned>(t.m_tiles);
       L.grid[1] = static_cast<unsigned>(t.n_tiles);
       L.grid[2] = static_cast<unsigned>(batch * t.splits);
+      L.cluster_z = static_cast<unsigned>(t.splits);
       L.smem = t.smem_bytes;
       return PASK_OK;
     }
@@ -444,14 +473,8 @@ PASK_API int pask_workspace_bytes(const pask_graph* g, uint64_t* bytes) {
   std::string err;
   int rc = extract_problems(g, &probs, &err);
   if (rc) return set_err(rc, err);
-  uint64_t need = 0;
-  for (size_t i = 0; i < probs.size(); ++i) {
-    int32_t M, N, K, batch, bm;
-    if (!contraction_shape(probs[i], g->nodes[i], &M, &N, &K, &batch, &bm)) continue;
-    const GemmTiling t = gemm_tiling(M, N, K, batch, bm);
-    if (t.splits > 1) need = std::max(need, (t.ws_counter_bytes + 255) / 256 * 256 + t.ws_partial_bytes);
-  }
-  *bytes = need;
+  // split-K partials are reduced on chip (cluster DSMEM): no global scratch today
+  *bytes = 0;
   return PASK_OK;
 }
 
@@ -558,9 +581,7 @@ PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, 
     if (outputs[i] && (rc = rebind(c, c->outputs[i], outputs[i]))) return rc;
   const Driver* d = c->d;
   CUstream s = static_cast<CUstream>(stream);
-  CUlaunchAttribute attr[1];
-  attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
-  attr[0].value.programmaticStreamSerializationAllowed = 1;
+  CUlaunchAttribute attr[2];
   for (size_t i = 0; i < c->launches.size(); ++i) {
     Launch& L = c->launches[i];
     if ((rc = wait_kernel(c, L.kernel))) return rc;
@@ -575,8 +596,21 @@ PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, 
     cfg.blockDimZ = L.block[2];
     cfg.sharedMemBytes = L.smem;
     cfg.hStream = s;
+    unsigned na = 0;
+    if (c->cfg.pdl && !c->cfg.instrument && i > 0) {
+      attr[na].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+      attr[na].value.programmaticStreamSerializationAllowed = 1;
+      ++na;
+    }
+    if (L.cluster_z > 1) {
+      attr[na].id = CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION;
+      attr[na].value.clusterDim.x = 1;
+      attr[na].value.clusterDim.y = 1;
+      attr[na].value.clusterDim.z = L.cluster_z;
+      ++na;
+    }
     cfg.attrs = attr;
-    cfg.numAttrs = (c->cfg.pdl && !c->cfg.instrument && i > 0) ? 1 : 0;
+    cfg.numAttrs = na;
     void* args[1] = {L.params.get()};
     const uint64_t t0 = now_ns();
     CUresult r = d->cuLaunchKernelEx(&cfg, c->fn[L.kernel], args, nullptr);
@@ -665,6 +699,17 @@ PASK_API int pask_kernel_is_loaded(const pask_ctx* c, int32_t k, int32_t* state)
   CUresult r = c->d->cuFuncIsLoaded(&ls, c->fn[k]);
   if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(c->d, r, "cuFuncIsLoaded"));
   *state = (ls == CU_FUNCTION_LOADING_STATE_LOADED) ? 1 : 0;
+  return PASK_OK;
+}
+
+PASK_API int pask_kernel_timeline(const pask_ctx* c, int32_t k, uint64_t* load_ns, uint64_t* ready_ns,
+                                  uint64_t* lib_ns) {
+  t_err.clear();
+  if (!c || k < 0 || k >= PASK_NUM_KERNELS) return set_err(PASK_EINVAL, "bad argument");
+  const bool done = c->ready[k].load(std::memory_order_acquire) == 1;
+  if (load_ns) *load_ns = done ? c->k_load_ns[k] : 0;
+  if (ready_ns) *ready_ns = (done && c->k_ready_at[k] > c->t_entry) ? c->k_ready_at[k] - c->t_entry : 0;
+  if (lib_ns) *lib_ns = done ? c->k_lib_ns[k] : 0;
   return PASK_OK;
 }
 

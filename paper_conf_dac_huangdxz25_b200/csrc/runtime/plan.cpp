@@ -354,44 +354,48 @@ bool contraction_shape(const Problem& p, const pask_node& nd, int32_t* M, int32_
   return false;
 }
 
-GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major) {
+GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma) {
   GemmTiling t{};
   t.M = M; t.N = N; t.K = K; t.batch = batch;
   constexpr int kSMs = 148;
+  // N tile: 16/32/48 for narrow outputs, else multiples of 64 (whole 128 B
+  // TMA boxes for the staged epilogue); MN-major B needs whole 64-wide boxes.
   if (b_major) {
     t.bn = std::min(256, (N + 63) / 64 * 64);
+  } else if (N <= 48) {
+    t.bn = (N + 15) / 16 * 16;
   } else {
-    t.bn = std::min(128, (N + 15) / 16 * 16);
+    t.bn = std::min(128, (N + 63) / 64 * 64);
   }
   t.m_tiles = (M + 127) / 128;
   t.n_tiles = (N + t.bn - 1) / t.bn;
-  // more CTAs for small-M layers: halve the N tile while the grid is far below one wave
-  while (!b_major && t.bn >= 128 && t.m_tiles * ((N + t.bn - 1) / t.bn) * batch < kSMs / 2) {
-    t.bn /= 2;
-    t.n_tiles = (N + t.bn - 1) / t.bn;
+  // more CTAs for small-M layers: halve a 128-wide N tile while far below one wave
+  if (!b_major && t.bn == 128 && static_cast<int64_t>(t.m_tiles) * t.n_tiles * batch < kSMs / 2) {
+    t.bn = 64;
+    t.n_tiles = (N + 63) / 64;
   }
   t.num_kb = (K + 63) / 64;
+  // split-K as a cluster of 2 / 4 / 8 CTAs (DSMEM reduction) when the grid is
+  // well below one wave and each split keeps >= 2 k-blocks
   const int64_t tiles = static_cast<int64_t>(t.m_tiles) * t.n_tiles * batch;
   int32_t splits = 1;
-  if (tiles < 100 && t.num_kb >= 4) {
-    splits = static_cast<int32_t>(std::min<int64_t>(kSMs / tiles, t.num_kb / 2));
-    splits = std::max(1, splits);
-  }
-  t.kb_per_split = (t.num_kb + splits - 1) / splits;
-  t.splits = (t.num_kb + t.kb_per_split - 1) / t.kb_per_split;
+  while (splits < 8 && tiles * splits * 2 <= kSMs && t.num_kb >= 4 * splits && t.bn <= 128) splits *= 2;
+  t.splits = splits;
+  t.rows_per = 128 / splits;
+  const int32_t kb_per = (t.num_kb + splits - 1) / splits;
   const uint32_t stage_bytes = 16384u + static_cast<uint32_t>(t.bn) * 128u;
-  int32_t stages = static_cast<int32_t>((200u * 1024u) / stage_bytes);
+  int32_t stages = static_cast<int32_t>((160u * 1024u) / stage_bytes);
   stages = std::min(stages, 8);
-  stages = std::min(stages, std::max(2, t.kb_per_split));
+  stages = std::min(stages, std::max(2, kb_per));
   t.stages = std::max(2, stages);
-  t.smem_bytes = t.stages * stage_bytes + (2 * t.stages + 1) * 8 + 8 + 1024;
+  const uint32_t ring = t.stages * stage_bytes;
+  const uint32_t stage32 = splits > 1 ? 128u * (t.bn + 4) * 4 : 0u;
+  const uint32_t reg0 = (std::max(ring, stage32) + 1023u) & ~1023u;
+  const uint32_t ro = c_tma ? ((128u * t.bn * 2 + 1023u) & ~1023u) : 0u;
+  t.smem_bytes = reg0 + ro + 1024u /*bias*/ + (2 * t.stages + 3) * 8u + 1024u /*align slack*/;
   uint32_t cols = 32;
   while (cols < static_cast<uint32_t>(t.bn)) cols <<= 1;
   t.tmem_cols = cols;
-  if (t.splits > 1) {
-    t.ws_partial_bytes = static_cast<uint64_t>(tiles) * t.splits * 128ull * t.bn * 4ull;
-    t.ws_counter_bytes = static_cast<uint64_t>(tiles) * 4ull;
-  }
   return t;
 }
 

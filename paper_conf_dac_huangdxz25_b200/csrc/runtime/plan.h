@@ -55,11 +55,11 @@ int execution_plan(const std::vector<Problem>& probs, const std::vector<int32_t>
 // the problem, so reuse stays bitwise reproducible).
 struct GemmTiling {
   int32_t M, N, K, batch;
-  int32_t bn, m_tiles, n_tiles, num_kb, kb_per_split, splits, stages;
+  int32_t bn, m_tiles, n_tiles, num_kb, splits, rows_per, stages;
   uint32_t smem_bytes, tmem_cols;
-  uint64_t ws_partial_bytes, ws_counter_bytes;
 };
-GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major);
+// c_tma: output / residual go through smem staging + TMA (changes the smem size)
+GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma);
 
 // Contraction view of a conv / GEMM problem (M, N, K, batch, b_major).
 bool contraction_shape(const Problem& p, const pask_node& node, int32_t* M, int32_t* N, int32_t* K,

@@ -77,7 +77,8 @@ class Stats(C.Structure):
 
 EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "pask_load_model",
            "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
-           "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name"]
+           "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name",
+           "pask_kernel_timeline"]
 
 _lib = None
 
@@ -105,6 +106,8 @@ def lib():
         "pask_stats": (C.c_int, [P, C.POINTER(Stats)]),
         "pask_kernel_is_loaded": (C.c_int, [P, C.c_int32, C.POINTER(C.c_int32)]),
         "pask_destroy": (C.c_int, [P]),
+        "pask_kernel_timeline": (C.c_int, [P, C.c_int32, C.POINTER(C.c_uint64),
+                                           C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
         "pask_last_error": (C.c_char_p, []),
         "pask_num_kernels": (C.c_int32, []),
         "pask_kernel_name": (C.c_char_p, [C.c_int32]),
@@ -190,6 +193,12 @@ class Context:
         v = C.c_int32()
         _check(lib().pask_kernel_is_loaded(self.h, k, C.byref(v)))
         return bool(v.value)
+
+    def kernel_timeline(self, k):
+        """(load_ns, ready_ns since load_model entry, lib_ns) of catalog kernel k."""
+        a, b, c = C.c_uint64(), C.c_uint64(), C.c_uint64()
+        _check(lib().pask_kernel_timeline(self.h, k, C.byref(a), C.byref(b), C.byref(c)))
+        return a.value, b.value, c.value
 
     def close(self):
         if self.h:

@@ -19,6 +19,10 @@ for name in sys.argv[1:]:
     errs = teacher_forced_errors(dm, spec, x)
     st = ctx.stats()
     print(f"== {name}: infer+sync {1e3*(t1-t0):.1f} ms  stats {st}")
+    for k in range(P.NUM_KERNELS):
+        ld, rd, lb = ctx.kernel_timeline(k)
+        if ld:
+            print(f"  load {P.kernel_name(k):16s} load {ld/1e3:8.1f} us  ready@ {rd/1e3:8.1f} us  lib {lb/1e3:8.1f} us")
     for (li, op, e), b in zip(errs, plan):
         L = spec["layers"][li]
         extra = ""
@@ -41,5 +45,6 @@ for name in sys.argv[1:]:
     ev1.record()
     torch.cuda.synchronize()
     print(f"== {name} hot {ev0.elapsed_time(ev1)/n:.3f} ms/inference")
-    ctx.close()
+    if os.environ.get("PASK_DEBUG_SKIP_CLOSE") != "1":
+        ctx.close()
     sys.stdout.flush()

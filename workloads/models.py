@@ -85,8 +85,10 @@ class _Builder:
         return self.tensors[t]
 
     # -- layers ---------------------------------------------------------
-    def layout(self, x, c_pad=8):
+    def layout(self, x, c_pad=None):
         n, c, h, w = self.shape(x)
+        if c_pad is None:
+            c_pad = max(8, (c + 7) // 8 * 8)
         y = self.tensor((n, c, h, w))
         self.layers.append(dict(op="layout", name=f"layout{len(self.layers)}", inputs=[x], out=y,
                                 c_pad=c_pad))
