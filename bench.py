@@ -1,0 +1,430 @@
+#!/usr/bin/env python
+"""PASK on B200 -- benchmark driver (one JSON line on rank 0).
+
+Workload (BASELINE.json configs[1]): ResNet-50, batch 1, 224x224, bf16, random
+weights, synthetic N(0,1) input.  A "step" is one inference through the C ABI
+(pask_infer: all 58 layers).  Per process:
+
+  cold   pask_load_model entry -> first inference complete (host clock; the
+         paper's cold start: planning + proactive code loading + issue + GPU)
+  hot    K timed inferences, L2 flushed before each (a 256 MiB memset outside
+         the CUDA-event window), mean device time per inference
+  value  imgs/s over all ranks = N * 1000 / max-over-ranks(hot ms)
+  e2e    the same through pask_infer_host: pinned host input -> H2D -> 58
+         kernels -> D2H of the softmax output -> sync, host clock per step
+
+N > 1 (torchrun): independent replicas, one process per GPU, cold-starting
+concurrently after a barrier (the path does not shard; no
+data-path collective -- gloo is used only for the barrier and the max).
+
+`--impl reference` times the fp64 numpy oracle (the reference arm of this
+tier) on the host cores, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "cold first-inference latency ms vs hot; imgs/s per B200; kernels loaded/model"
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured"
+    return PEAKS_FALLBACK, "fallback"
+
+
+# ---------------------------------------------------------------- algorithmic work
+def node_work(spec, li):
+    """(bytes, flops) of layer li: inputs + weights + outputs (+ residual, bias)
+    at their device precision (bf16 tensors, fp32 bias), SURVEY.md §8(d)."""
+    L = spec["layers"][li]
+    sh = spec["tensors"]
+    op = L["op"]
+
+    def numel(name):
+        n = 1
+        for d in sh[name]:
+            n *= d
+        return n
+    if op == "layout":
+        n, c, h, w = sh[L["inputs"][0]]
+        return n * c * h * w * 4 + n * h * w * L["c_pad"] * 2, 0
+    if op == "conv":
+        k, cg, r, s = L["w"].shape
+        n, c, h, w = sh[L["inputs"][0]]
+        c_dev = max(8, (c + 7) // 8 * 8) if L["groups"] == 1 else c
+        _, _, p, q = sh[L["out"]]
+        byt = n * h * w * c_dev * 2 + k * r * s * (c_dev if L["groups"] == 1 else 1) * 2 + \
+            n * p * q * k * 2 + (k * 4 if L["b"] is not None else 0)
+        if L["res"]:
+            byt += n * p * q * k * 2
+        flops = 2 * n * p * q * k * (c_dev if L["groups"] == 1 else 1) * r * s
+        return byt, flops
+    if op == "linear":
+        m, nout = sh[L["out"]]
+        kin = L["w"].shape[1]
+        byt = m * kin * 2 + nout * kin * 2 + m * nout * 2 + (nout * 4 if L["b"] is not None else 0)
+        if L["res"]:
+            byt += m * nout * 2
+        return byt, 2 * m * nout * kin
+    if op == "pool":
+        return numel(L["inputs"][0]) * 2 + numel(L["out"]) * 2, 0
+    return numel(L["inputs"][0]) * 2 + numel(L["out"]) * 2, 0
+
+
+# ---------------------------------------------------------------- replicas
+def reduce_max(values, dist=None):
+    """Element-wise max over ranks (gloo all_reduce on CPU; no data-path
+    collective: replicas share nothing but this timing reduction)."""
+    import torch
+    t = torch.tensor([float(v) for v in values], dtype=torch.float64)
+    if dist is not None:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return [float(v) for v in t]
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    def __init__(self, device):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                       "-lms", "50", "-i", str(device)],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        out, _ = self.p.communicate(timeout=10)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- reference arm / cpu baseline
+def time_oracle(spec, x, max_steps, budget_s):
+    """The fp64 numpy oracle, as it stands, full forwards of one image."""
+    from oracle import models as om
+    times = []
+    t_end = time.perf_counter() + budget_s
+    for _ in range(max_steps):
+        t0 = time.perf_counter()
+        om.run_model(spec, x)
+        times.append(time.perf_counter() - t0)
+        if time.perf_counter() > t_end:
+            break
+    return times
+
+
+def cores_used():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count()
+
+
+def run_reference(args, spec, x, rank):
+    if rank != 0:
+        return
+    w = time_oracle(spec, x, max(args.warmup, 0), 60.0) if args.warmup else []
+    ts = time_oracle(spec, x, args.steps, 240.0)
+    mean_s = statistics.mean(ts)
+    val = 1.0 / mean_s
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "imgs/s",
+        "n_gpus": args.gpus, "steps": len(ts), "warmup": len(w), "ms_per_step": round(1e3 * mean_s, 2),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": {"workload": args.workload_name, "global_batch": 1,
+                                        "model": args.model},
+        "cpu_baseline": {"value": round(val, 4), "unit": "imgs/s", "cores": cores_used(),
+                         "kind": "oracle",
+                         "sample": f"{len(ts)} full fp64 numpy-oracle forwards of one image"},
+        "e2e": {"value": round(val, 4), "unit": "imgs/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="pask", choices=["pask", "reference"])
+    ap.add_argument("--model", default="resnet50",
+                    choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
+    ap.add_argument("--packaging", type=int, default=0, choices=[0, 1],
+                    help="0: one code object per kernel (default); 1: whole catalog in one")
+    args = ap.parse_args()
+    args.workload_name = {
+        "tiny_cnn": "tiny CNN 3xconv3x3(16/32/64)+maxpool+FC, 32x32x3, batch 1, bf16",
+        "resnet50": "ResNet-50 batch 1 224x224 cold start, all convs served by one reused "
+                    "implicit-GEMM kernel",
+        "mobilenet_v2": "MobileNetV2 batch 1 224x224 (depthwise + pointwise convs) cold start",
+        "bert_base": "BERT-base seq 128 batch 1 (GEMM + softmax + layernorm) cold start",
+    }[args.model]
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+
+    from workloads import build_model
+    spec, x = build_model(args.model)
+
+    if args.impl == "reference":
+        run_reference(args, spec, x, rank)
+        if dist:
+            dist.destroy_process_group()
+        return
+
+    import torch
+
+    from paper_conf_dac_huangdxz25_b200 import build as pbuild
+    from paper_conf_dac_huangdxz25_b200 import pask as P
+    from paper_conf_dac_huangdxz25_b200.model import DeviceModel
+
+    pbuild.build()
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    stream = torch.cuda.current_stream(dev)
+    sp = stream.cuda_stream
+    dm = DeviceModel(spec, device=dev)
+    dm.set_input(x)
+    flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def flush():
+        flush_buf.zero_()
+
+    flush()
+    torch.cuda.synchronize()
+    ctx = P.Context(local_rank, P.config(packaging=args.packaging))
+    n_nodes = len(spec["layers"])
+
+    def barrier():
+        if dist:
+            dist.barrier()
+
+    # ---------------- cold: pask_load_model entry -> first inference done
+    barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter_ns()
+    plan = ctx.load_model(dm.graph)
+    ctx.infer(sp)
+    ctx.sync()
+    t1 = time.perf_counter_ns()
+    cold_ms = (t1 - t0) / 1e6
+    cold_stats = ctx.stats()
+    timeline = {}
+    for k in range(P.NUM_KERNELS):
+        ld, rd, lb = ctx.kernel_timeline(k)
+        if ld:
+            timeline[P.kernel_name(k)] = {"load_us": round(ld / 1e3, 1), "ready_at_us": round(rd / 1e3, 1),
+                                          "lib_us": round(lb / 1e3, 1)}
+    loaded = sorted(P.kernel_name(k) for k in range(P.NUM_KERNELS) if ctx.kernel_is_loaded(k))
+
+    # ---------------- warmup
+    for _ in range(args.warmup):
+        flush()
+        ctx.infer(sp)
+    torch.cuda.synchronize()
+
+    # ---------------- timed: K steps, L2 flushed between steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    sampler = ClockSampler(local_rank)
+    time.sleep(0.2)
+    barrier()
+    torch.cuda.synchronize()
+    w0 = time.perf_counter()
+    for i in range(args.steps):
+        if not args.no_flush:
+            flush()
+        ev[i][0].record(stream)
+        ctx.infer(sp)
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    w1 = time.perf_counter()
+    barrier()
+    clocks = sampler.stop()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    hot_ms = statistics.mean(step_ms)
+
+    # ---------------- L2-warm back-to-back (context: serving the same model repeatedly)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    nw = max(20, args.steps // 2)
+    for _ in range(nw):
+        ctx.infer(sp)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    hot_warm_ms = e0.elapsed_time(e1) / nw
+
+    # ---------------- e2e through the public API with host buffers
+    in_host = torch.from_numpy(x.astype("float32")).pin_memory()
+    out_name = spec["outputs"][0]
+    out_dev = dm.t[out_name]
+    out_host = torch.empty(out_dev.shape, dtype=out_dev.dtype).pin_memory()
+    h2d = in_host.numel() * in_host.element_size()
+    d2h = out_host.numel() * out_host.element_size()
+    e2e_s = []
+    for i in range(args.warmup + args.steps):
+        if not args.no_flush:
+            flush()
+        torch.cuda.synchronize()
+        a = time.perf_counter()
+        ctx.infer_host([in_host.data_ptr()], [out_host.data_ptr()], sp)
+        b = time.perf_counter()
+        if i >= args.warmup:
+            e2e_s.append(b - a)
+    e2e_ms = 1e3 * statistics.mean(e2e_s)
+
+    # ---------------- per-kernel roofline: instrumented pass (separate context)
+    ictx = P.Context(local_rank, P.config(instrument=1))
+    iplan = ictx.load_model(dm.graph)
+    reps = 10
+    acc = [0] * n_nodes
+    for r in range(reps + 2):
+        flush()
+        ictx.infer(sp)
+        ictx.sync()
+        if r >= 2:
+            acc = [a + b for a, b in zip(acc, ictx.node_times())]
+    node_ms = [a / reps / 1e6 for a in acc]
+    ictx.close()
+    per_kernel = {}
+    for (i, want, bound, how, lk), t in zip(plan, node_ms):
+        byt, fl = node_work(spec, i)
+        d = per_kernel.setdefault(P.kernel_name(bound), {"launches": 0, "ms": 0.0, "bytes": 0, "flops": 0})
+        d["launches"] += 1
+        d["ms"] += t
+        d["bytes"] += byt
+        d["flops"] += fl
+    dom = max(per_kernel, key=lambda k: per_kernel[k]["ms"])
+    peaks, peak_src = load_peaks()
+    dk = per_kernel[dom]
+    gbs = dk["bytes"] / (dk["ms"] * 1e-3) / 1e9
+    tfl = dk["flops"] / (dk["ms"] * 1e-3) / 1e12
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "dram_traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as f:
+            traffic = json.load(f).get(args.model, {}).get(dom)
+    roofline = {"bound": "hbm", "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": traffic,
+                "kernel": dom, "launches_per_step": dk["launches"],
+                "algorithmic_bytes_per_launch": int(dk["bytes"] / dk["launches"]),
+                "avg_launch_us": round(1e3 * dk["ms"] / dk["launches"], 2),
+                "tensor_tflops": round(tfl, 2),
+                "tensor_frac_of_bf16_burst": round(tfl / peaks["bf16_tflops"], 4),
+                "peak_source": f"{peak_src} (MEASURED_PEAKS.json hbm_gbs / bf16_tflops)",
+                "l2": "flushed before each inference (weights from HBM)"}
+
+    # ---------------- max over ranks
+    hot_max, cold_max, e2e_max, warm_max = reduce_max([hot_ms, cold_ms, e2e_ms, hot_warm_ms], dist)
+    ctx.close()
+    if rank != 0:
+        if dist:
+            dist.destroy_process_group()
+        return
+
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        ts = time_oracle(spec, x, 5, 20.0)
+        cpu = {"value": round(1.0 / statistics.mean(ts), 4), "unit": "imgs/s", "cores": cores_used(),
+               "kind": "oracle",
+               "sample": f"{len(ts)} full fp64 numpy-oracle forwards of one {args.model} image"}
+
+    st = cold_stats
+    line = {
+        "metric": METRIC,
+        "value": round(world * 1000.0 / hot_max, 2),
+        "unit": "imgs/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(hot_max, 4),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "bf16",
+        "data": "synthetic (seeded N(0,1) input, random-init weights of the architecture)",
+        "config": {"workload": args.workload_name, "model": args.model, "global_batch": world,
+                   "per_gpu_batch": 1, "parallelism": f"replicas{world}",
+                   "packaging": ["one code object per kernel", "single code object"][args.packaging],
+                   "l2": "warm (no flush)" if args.no_flush else
+                         "flushed (256 MiB memset) before every timed inference"},
+        "cold_ms": round(cold_max, 3),
+        "hot_ms": round(hot_max, 4),
+        "cold_over_hot": round(cold_max / hot_max, 3),
+        "hot_l2_warm_ms": round(warm_max, 4),
+        "kernels_loaded": st["kernels_loaded"],
+        "kernels_loaded_names": loaded,
+        "code_objects_loaded": st["code_objects_loaded"],
+        "plan": {"queries": st["queries"], "hits": st["hits"], "lookups": st["lookups"],
+                 "reused_nodes": sum(1 for b in plan if b[3] == 1)},
+        "cold_breakdown_us": {"plan": round(st["plan_ns"] / 1e3, 1),
+                              "encode": round(st["encode_ns"] / 1e3, 1),
+                              "load_total": round(st["load_ns"] / 1e3, 1),
+                              "load_exposed": round(st["load_exposed_ns"] / 1e3, 1),
+                              "issue": round(st["issue_ns"] / 1e3, 1),
+                              "gpu_span": round(st["gpu_span_ns"] / 1e3, 1),
+                              "cold_wall": round(st["cold_wall_ns"] / 1e3, 1)},
+        "load_timeline_us": timeline,
+        "per_kernel_ms": {k: round(v["ms"], 4) for k, v in per_kernel.items()},
+        "e2e": {"value": round(world * 1000.0 / e2e_max, 2), "unit": "imgs/s",
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "ms_per_step": round(e2e_max, 4)},
+        "gpu_launches": n_nodes * args.steps,
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "clocks": clocks,
+        "wall_s_timed_region": round(w1 - w0, 4),
+    }
+    print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

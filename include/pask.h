@@ -173,6 +173,9 @@ typedef struct {
   int32_t proactive;  /* 1 = loader thread; 0 = reactive load at first launch   */
   int32_t pdl;        /* 1 = programmatic dependent launch between consecutive kernels        */
   int32_t instrument; /* 1 = per-node CUDA events for gpu_busy_ns (perturbs timing)           */
+  int32_t packaging;  /* 0 = one code object per catalog kernel (default: a load costs ~0.9 us
+                         per KB of image, so only the bound kernels' code is parsed);
+                         1 = the whole catalog as one code object                            */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;
@@ -266,6 +269,11 @@ int pask_kernel_is_loaded(const pask_ctx *ctx, int32_t kernel_id, int32_t *state
  *   lib_ns      cuLibraryLoadData time if this kernel's load performed it. */
 int pask_kernel_timeline(const pask_ctx *ctx, int32_t kernel_id, uint64_t *load_ns,
                          uint64_t *ready_ns, uint64_t *lib_ns);
+
+/* Per-node GPU durations (ns) of the last inference issued with
+ * cfg.instrument = 1 (call pask_sync first).  ns_out: caller array of
+ * n_nodes entries; PASK_ESTATE if the context is not instrumented. */
+int pask_node_times(const pask_ctx *ctx, uint64_t *ns_out, int32_t n_nodes);
 
 /* Join the loader thread, unload the library and free host state. */
 int pask_destroy(pask_ctx *ctx);

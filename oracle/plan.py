@@ -54,7 +54,8 @@ def is_applicable(kid, p):
     """IsApplicable(kernel, problem) -- PAPER.md:83, Alg. 1 l.15."""
     op = p["op"]
     if kid == K_LAYOUT:
-        return op == LAYOUT and p["k"] % 8 == 0 and p["c"] <= p["k"]
+        return (op == LAYOUT and p["k"] % 8 == 0 and p["c"] <= p["k"]
+                and p["n"] * p["h"] * p["w"] * max(p["c"], p["k"]) < 2 ** 31)
     if kid == K_IGEMM:
         return (op == CONV and p["groups"] == 1 and p["c"] % 8 == 0 and p["k"] % 8 == 0
                 and 1 <= p["r"] <= 16 and 1 <= p["s"] <= 16
@@ -68,12 +69,14 @@ def is_applicable(kid, p):
                 and p["pad_h"] == 0 and p["pad_w"] == 0
                 and p["c"] % 8 == 0 and p["k"] % 8 == 0)
     if kid == K_DW:
-        return (op == DWCONV and p["c"] % 8 == 0 and 1 <= p["r"] <= 15 and 1 <= p["s"] <= 15
+        return (op == DWCONV and p["c"] % 8 == 0 and p["n"] * p["h"] * p["w"] * p["c"] < 2 ** 31
+                and 1 <= p["r"] <= 15 and 1 <= p["s"] <= 15
                 and 1 <= p["stride_h"] <= 8 and 1 <= p["stride_w"] <= 8
                 and 1 <= p["dil_h"] <= 8 and 1 <= p["dil_w"] <= 8
                 and p["p"] >= 1 and p["q"] >= 1)
     if kid == K_POOL:
-        return (op == POOL and p["c"] % 8 == 0 and p["r"] * p["s"] <= 1024
+        return (op == POOL and p["c"] % 8 == 0 and p["n"] * p["h"] * p["w"] * p["c"] < 2 ** 31
+                and p["r"] * p["s"] <= 1024
                 and p["stride_h"] >= 1 and p["stride_w"] >= 1
                 and p["pad_h"] < p["r"] and p["pad_w"] < p["s"])
     if kid == K_GAVG:
@@ -119,8 +122,9 @@ _ZERO = dict(op=0, n=0, h=0, w=0, c=0, k=0, r=0, s=0, stride_h=0, stride_w=0, pa
 
 def problems_from_spec(spec):
     """Extract the problem p_i of every spec layer (parse step P_i).
-    Image tensors are NHWC on the device with C padded to a multiple of 8 only
-    for the layout output (the stem input)."""
+    Problems are stated on the device tensors (reading D1): the layout
+    output carries C padded to c_pad; a pool keeps its input's (padded) channel
+    count; a conv output has K channels; a flattened FC reduces over H*W*C_dev."""
     shapes = spec["tensors"]
     devc = {}
     out = []
@@ -144,6 +148,8 @@ def problems_from_spec(spec):
             p["op"] = _conv_class(p)
         elif op == "pool":
             n, c, h, w = shapes[layer["inputs"][0]]
+            c = devc.get(layer["inputs"][0], c)
+            devc[layer["out"]] = c
             _, _, pp, qq = shapes[layer["out"]]
             p.update(op=POOL, n=n, h=h, w=w, c=c, k=c, r=layer["kernel"][0],
                      s=layer["kernel"][1], stride_h=layer["stride"][0],
@@ -153,6 +159,10 @@ def problems_from_spec(spec):
         elif op == "linear":
             m, nout = shapes[layer["out"]]
             kin = layer["w"].shape[1]
+            src = layer["inputs"][0]
+            if len(shapes[src]) == 4:        # flattened image: K over the device channels
+                _, c, h, w = shapes[src]
+                kin = h * w * devc.get(src, c)
             p.update(op=GEMM, gm=m, gn=nout, gk=kin, batch=1, lda=kin, ldb=kin)
         elif op == "qk":
             s_, three_h = shapes[layer["inputs"][0]]

@@ -24,10 +24,12 @@
 //   epilogue  : TMEM -> registers -> (+bias, +residual from smem, act) -> bf16
 //               staged in smem -> TMA tensor store (clips the M / N tails)
 //   split-K   : a thread-block cluster of S = 2/4/8 CTAs along z, one K range
-//               each; every CTA parks its fp32 tile in its own smem, then rank
-//               r reduces rows [r*128/S, (r+1)*128/S) over the S peers through
-//               DSMEM in fixed rank order 0..S-1 -- deterministic, so a given
-//               (kernel, problem) is bitwise reproducible (SURVEY.md §7 part 8).
+//               each; rank r owns rows [r*128/S, (r+1)*128/S) of the tile.  Every
+//               CTA pushes each fp32 row of its partial to the owner's receive
+//               slot [source rank] (st.async into DSMEM, completion counted on the
+//               owner's mbarrier); the owner sums its S slots in fixed rank order
+//               0..S-1 -- deterministic, so a given (kernel, problem) is bitwise
+//               reproducible (SURVEY.md §7 part 8) -- and runs the epilogue.
 #pragma once
 #include "pask_params.h"
 #include "ptx.cuh"
@@ -136,9 +138,10 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const uint32_t b_bytes = static_cast<uint32_t>(bn) * kBK * 2;
   const uint32_t stage_bytes = kABytes + b_bytes;
   // ---- smem carve-up (mirrors gemm_tiling() on the host)
-  const uint32_t ring_bytes = stages * stage_bytes;
-  const uint32_t stage32_pitch = (bn + 4) * 4;  // fp32 split-K staging row pitch (bank spread)
-  const uint32_t reg0 = (max(ring_bytes, splits > 1 ? 128u * stage32_pitch : 0u) + 1023u) & ~1023u;
+  const uint32_t ring_bytes = (stages * stage_bytes + 1023u) & ~1023u;
+  const uint32_t recv_pitch = (bn + 4) * 4;  // fp32 split-K receive row pitch (bank spread)
+  const uint32_t recv_bytes = splits > 1 ? ((128u * recv_pitch + 1023u) & ~1023u) : 0u;
+  const uint32_t reg0 = ring_bytes + recv_bytes;
   const uint32_t ro_bytes = p.c_tma ? ((128u * bn * 2 + 1023u) & ~1023u) : 0u;
   float* s_bias = reinterpret_cast<float*>(smem + reg0 + ro_bytes);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + reg0 + ro_bytes + 1024);
@@ -147,8 +150,10 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const uint32_t empty0 = smem_u32(bars + stages);
   const uint32_t accum_bar = smem_u32(bars + 2 * stages);
   const uint32_t res_bar = smem_u32(bars + 2 * stages + 1);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * stages + 2);
+  const uint32_t recv_bar = smem_u32(bars + 2 * stages + 2);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * stages + 3);
   const uint32_t ro = smem_base + reg0;
+  const uint32_t recv = smem_base + ring_bytes;  // slot s: rows [s*rows_per, (s+1)*rows_per)
 
   const bool gather = kAllowGather && (p.a_mode == A_GATHER);
   const int mt = blockIdx.x, nt = blockIdx.y;
@@ -162,6 +167,9 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int rows_per = p.rows_per;
   const int r0 = splits > 1 ? static_cast<int>(cluster_ctarank()) * rows_per : 0;
   const bool res_tma = p.c_tma && p.res != nullptr;
+  unsigned long long* trace =
+      p.trace ? p.trace + 8ull * (blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) : nullptr;
+  if (trace && t == 0) trace[0] = globaltimer();
 
   // ---------------- prologue (overlaps the previous kernel under PDL)
   if (t == 0) {
@@ -171,6 +179,9 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
     }
     mbar_init(accum_bar, 1u);
     mbar_init(res_bar, 1u);
+    mbar_init(recv_bar, 1u);
+    if (splits > 1)  // the S-1 peers push rows_per x bn fp32 each into this CTA
+      mbar_arrive_expect_tx(recv_bar, static_cast<uint32_t>((splits - 1) * rows_per * bn * 4));
     fence_barrier_init();
   }
   if (warp == 4 && lane == 0) {
@@ -183,23 +194,27 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
+  if (splits > 1) cluster_sync_all();  // peers' receive barriers are initialised
   const uint32_t tmem_base = *tmem_slot;
+  if (trace && t == 0) trace[1] = globaltimer();
 
   pdl_wait();               // inputs of this layer are complete and visible
   pdl_launch_dependents();  // let the next layer's prologue start
+  if (trace && t == 0) trace[2] = globaltimer();
 
   if (warp == 4) {
     // ================= TMA producer
     if (lane == 0) {
       if (res_tma) {  // residual rows [r0, r0 + rows_per) of the tile, consumed by the epilogue
         mbar_arrive_expect_tx(res_bar, static_cast<uint32_t>(rows_per * bn * 2));
+#pragma unroll 1
         for (int j = 0; j < bn / box_cols; ++j)
           tma_load_3d(ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), &p.tmap_r, res_bar,
                       n0 + j * box_cols, m0 + r0, b);
       }
+      int s = 0;
+      uint32_t ph = 0;
       for (int i = 0; i < nk; ++i) {
-        const int s = i % stages;
-        const uint32_t ph = (i / stages) & 1;
         mbar_wait(empty0 + 8 * s, ph ^ 1);
         const uint32_t sa = smem_base + s * stage_bytes;
         const uint32_t sb = sa + kABytes;
@@ -209,8 +224,13 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         if (p.b_major == 0) {
           tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
         } else {
+#pragma unroll 1
           for (int j = 0; j < bn / 64; ++j)
             tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * s, n0 + j * 64, kb * kBK, b);
+        }
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1;
         }
       }
     }
@@ -218,11 +238,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   } else if (warp == 5) {
     // ================= MMA issuer (one thread issues for the whole CTA)
     if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0;
       for (int i = 0; i < nk; ++i) {
-        const int s = i % stages;
-        const uint32_t ph = (i / stages) & 1;
         mbar_wait(full0 + 8 * s, ph);
         tc_fence_after();
+        if (trace && i == 0) trace[3] = globaltimer();
         const uint32_t sa = smem_base + s * stage_bytes;
         const uint32_t sb = sa + kABytes;
 #pragma unroll
@@ -236,8 +257,13 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           umma_f16(tmem_base, adesc, bdesc, p.idesc, (i | k) != 0 ? 1u : 0u);
         }
         umma_commit(empty0 + 8 * s);  // frees the smem slot when these MMAs complete
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1;
+        }
       }
       umma_commit(accum_bar);  // accumulator complete -> epilogue
+      if (trace) trace[4] = globaltimer();
     }
     __syncwarp();
   } else {
@@ -250,19 +276,29 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x);
       int ih0[8], iw0[8], nb[8];
       bool rv[8];
-      const int pq = p.P * p.Q;
+      {
+        // output pixel of row rg, then step 16 pixels per ri (no per-row divisions)
+        const int m = m0 + rg;
+        const int pq = p.P * p.Q;
+        int n = m / pq;
+        const int rem = m - n * pq;
+        int pp = rem / p.Q;
+        int qq = rem - pp * p.Q;
 #pragma unroll
-      for (int ri = 0; ri < 8; ++ri) {
-        const int m = m0 + rg + 16 * ri;
-        rv[ri] = m < p.M;
-        const int mm = rv[ri] ? m : 0;
-        const int n = mm / pq;
-        const int rem = mm - n * pq;
-        const int pp = rem / p.Q;
-        const int qq = rem - pp * p.Q;
-        ih0[ri] = pp * p.sh - p.ph;
-        iw0[ri] = qq * p.sw - p.pw;
-        nb[ri] = n * p.H;
+        for (int ri = 0; ri < 8; ++ri) {
+          rv[ri] = (m + 16 * ri) < p.M;
+          ih0[ri] = pp * p.sh - p.ph;
+          iw0[ri] = qq * p.sw - p.pw;
+          nb[ri] = n * p.H;
+          qq += 16;
+          while (qq >= p.Q) {
+            qq -= p.Q;
+            if (++pp == p.P) {
+              pp = 0;
+              ++n;
+            }
+          }
+        }
       }
       int kk = kb_begin * kBK + 8 * j;
       int tap = kk / p.C;
@@ -270,9 +306,9 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       int r = tap / p.S;
       int s = tap - r * p.S;
       const int lag = min(2, stages - 1);
+      int st = 0, st_lag = 0;  // ring slot being filled / being published
+      uint32_t ph = 0;
       for (int i = 0; i < nk; ++i) {
-        const int st = i % stages;
-        const uint32_t ph = (i / stages) & 1;
         mbar_wait(empty0 + 8 * st, ph ^ 1);
         const uint32_t sa = smem_base + st * stage_bytes;
         const bool kval = kk < p.K;
@@ -292,7 +328,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         if (i >= lag) {
           cp_async_wait_dyn(lag);
           fence_proxy_async_smem();  // generic-proxy smem writes -> tcgen05 (async proxy)
-          mbar_arrive(full0 + 8 * ((i - lag) % stages));
+          mbar_arrive(full0 + 8 * st_lag);
+          if (++st_lag == stages) st_lag = 0;
+        }
+        if (++st == stages) {
+          st = 0;
+          ph ^= 1;
         }
         kk += kBK;
         c += kBK;
@@ -306,33 +347,46 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       }
       cp_async_wait<0>();
       fence_proxy_async_smem();
-      for (int i = max(0, nk - lag); i < nk; ++i) mbar_arrive(full0 + 8 * (i % stages));
+      for (int i = max(0, nk - lag); i < nk; ++i) {
+        mbar_arrive(full0 + 8 * st_lag);
+        if (++st_lag == stages) st_lag = 0;
+      }
     }
     named_bar_sync(1, 128);  // s_bias complete
     mbar_wait(accum_bar, 0);
     tc_fence_after();
+    if (trace && t == 0) trace[5] = globaltimer();
   }
 
   // ---------------- epilogue
   EpiCtx e{s_bias, ro, box_cols, m0, n0, b};
   const uint32_t taddr = tmem_base + (static_cast<uint32_t>((warp & 3) * 32) << 16);
   const int cpr = bn >> 4;  // 16-column chunks per row
-  if (splits > 1) {
-    // park this split's fp32 tile in smem (ring is idle: all MMAs completed)
-    if (warp < 4) {
-      const int row = warp * 32 + lane;
-      const uint32_t dst = smem_base + row * stage32_pitch;
-      for (int cb = 0; cb < bn; cb += 16) {
-        float v[16];
-        tmem_ld16(taddr + cb, v);
+  if (splits > 1 && warp < 4) {
+    // push this split's fp32 rows to their owners' receive slot [my rank]
+    const int row = warp * 32 + lane;
+    const uint32_t owner = static_cast<uint32_t>(row / rows_per);
+    const uint32_t me = cluster_ctarank();
+    const uint32_t slot_row = me * rows_per + (row - owner * rows_per);
+    const uint32_t local = recv + slot_row * recv_pitch;
+    const uint32_t remote = mapa_cluster(local, owner);
+    const uint32_t rbar = mapa_cluster(recv_bar, owner);
+    for (int cb = 0; cb < bn; cb += 16) {
+      float v[16];
+      tmem_ld16(taddr + cb, v);
 #pragma unroll
-        for (int q4 = 0; q4 < 4; ++q4)
-          asm volatile("st.shared.v4.f32 [%0], {%1,%2,%3,%4};" ::"r"(dst + (cb + 4 * q4) * 4),
+      for (int q4 = 0; q4 < 4; ++q4) {
+        if (owner == me)
+          asm volatile("st.shared.v4.f32 [%0], {%1,%2,%3,%4};" ::"r"(local + (cb + 4 * q4) * 4),
                        "f"(v[4 * q4]), "f"(v[4 * q4 + 1]), "f"(v[4 * q4 + 2]), "f"(v[4 * q4 + 3])
                        : "memory");
+        else
+          st_async_f4(remote + (cb + 4 * q4) * 4, v[4 * q4], v[4 * q4 + 1], v[4 * q4 + 2], v[4 * q4 + 3],
+                      rbar);
       }
     }
-    cluster_sync_all();  // every split's partial tile is parked
+    named_bar_sync(1, 128);  // own-slot rows visible to all epilogue threads
+    mbar_wait(recv_bar, 0);  // every peer's rows have landed
   }
   if (warp < 4) {
     if (res_tma) mbar_wait(res_bar, 0);
@@ -348,37 +402,45 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         tmem_ld16(taddr + cb, v);  // warp-collective
       } else {
         const int it = t + 128 * k;
-        row = r0 + it / cpr;
-        cb = (it - (it / cpr) * cpr) << 4;
-        const uint32_t local = smem_base + row * stage32_pitch + cb * 4;
+        const int lr = it / cpr;  // row within this rank's slice
+        row = r0 + lr;
+        cb = (it - lr * cpr) << 4;
+        const uint32_t src = recv + lr * recv_pitch + cb * 4;
 #pragma unroll
         for (int i = 0; i < 16; ++i) v[i] = 0.f;
         for (int sp = 0; sp < splits; ++sp) {  // fixed rank order: deterministic
-          const uint32_t ra = mapa_cluster(local, static_cast<uint32_t>(sp));
+          const uint32_t a = src + sp * rows_per * recv_pitch;
+          float4 f[4];
+#pragma unroll
+          for (int q4 = 0; q4 < 4; ++q4)
+            asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
+                         : "=f"(f[q4].x), "=f"(f[q4].y), "=f"(f[q4].z), "=f"(f[q4].w)
+                         : "r"(a + 16 * q4));
 #pragma unroll
           for (int q4 = 0; q4 < 4; ++q4) {
-            const float4 f = ld_dsmem_f4(ra + 16 * q4);
-            v[4 * q4] += f.x;
-            v[4 * q4 + 1] += f.y;
-            v[4 * q4 + 2] += f.z;
-            v[4 * q4 + 3] += f.w;
+            v[4 * q4] += f[q4].x;
+            v[4 * q4 + 1] += f[q4].y;
+            v[4 * q4 + 2] += f[q4].z;
+            v[4 * q4 + 3] += f[q4].w;
           }
         }
       }
       epi16(p, e, row, cb, v);
     }
   }
+  if (trace && t == 0) trace[6] = globaltimer();
   if (p.c_tma && warp < 4) {
     fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
     named_bar_sync(1, 128);
     if (t == 0) {
+#pragma unroll 1
       for (int j = 0; j < bn / box_cols; ++j)
         tma_store_3d(&p.tmap_c, ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), n0 + j * box_cols,
                      m0 + r0, b);
       tma_store_commit_and_wait_read();
     }
   }
-  if (splits > 1) cluster_sync_all();  // peers finished reading this CTA's partial tile
+  if (trace && t == 0) trace[7] = globaltimer();
 
   // ---------------- teardown
   tc_fence_before();

@@ -25,15 +25,15 @@ __device__ __forceinline__ float warp_max(float v) {
 __device__ __forceinline__ void layout_body(const LayoutParams& p) {
   pdl_wait();
   pdl_launch_dependents();
+  // 32-bit indices: the planner guarantees n*h*w*c_out < 2^31
   const int chunks = p.c_out >> 3;
-  const int64_t hw = static_cast<int64_t>(p.h) * p.w;
-  const int64_t total = static_cast<int64_t>(p.n) * hw * chunks;
-  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < total;
-       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
-    const int64_t pix = idx / chunks;
-    const int ch = static_cast<int>(idx - pix * chunks);
-    const int64_t n = pix / hw;
-    const int64_t off = pix - n * hw;
+  const int hw = p.h * p.w;
+  const int total = p.n * hw * chunks;
+  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
+    const int pix = idx / chunks;
+    const int ch = idx - pix * chunks;
+    const int n = pix / hw;
+    const int off = pix - n * hw;
     float f[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
@@ -52,23 +52,23 @@ __device__ __forceinline__ void layout_body(const LayoutParams& p) {
 __device__ __forceinline__ void pool_body(const PoolParams& p) {
   pdl_wait();
   pdl_launch_dependents();
+  // 32-bit indices: the planner guarantees n*H*W*C < 2^31
   const int chunks = p.C >> 3;
-  const int64_t total = static_cast<int64_t>(p.n) * p.P * p.Q * chunks;
+  const int total = p.n * p.P * p.Q * chunks;
   const uint4* x = reinterpret_cast<const uint4*>(p.x);
   const int lane = threadIdx.x & 31;
-  const int64_t first = p.per_warp ? (blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x) >> 5
-                                   : blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
-  const int64_t step = p.per_warp ? (static_cast<int64_t>(gridDim.x) * blockDim.x) >> 5
-                                  : static_cast<int64_t>(gridDim.x) * blockDim.x;
+  const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
+  const int first = p.per_warp ? (gtid >> 5) : gtid;
+  const int step = p.per_warp ? ((gridDim.x * blockDim.x) >> 5) : gridDim.x * blockDim.x;
   const int taps = p.R * p.S;
-  for (int64_t idx = first; idx < total; idx += step) {
-    int64_t t = idx;
-    const int ch = static_cast<int>(t % chunks);
+  for (int idx = first; idx < total; idx += step) {
+    int t = idx;
+    const int ch = t % chunks;
     t /= chunks;
-    const int q = static_cast<int>(t % p.Q);
+    const int q = t % p.Q;
     t /= p.Q;
-    const int pp = static_cast<int>(t % p.P);
-    const int n = static_cast<int>(t / p.P);
+    const int pp = t % p.P;
+    const int n = t / p.P;
     float acc[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = p.mode == 0 ? -INFINITY : 0.f;
@@ -79,7 +79,7 @@ __device__ __forceinline__ void pool_body(const PoolParams& p) {
       const int ih = ih0 + r, iw = iw0 + s;
       if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;
       float f[8];
-      unpack_bf16x8(__ldg(x + ((static_cast<int64_t>(n) * p.H + ih) * p.W + iw) * chunks + ch), f);
+      unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), f);
       cnt += 1.f;
       if (p.mode == 0) {
 #pragma unroll
@@ -151,19 +151,19 @@ __device__ __forceinline__ void gavg_body(const PoolParams& p) {
 __device__ __forceinline__ void dw_body(const DwParams& p) {
   pdl_wait();
   pdl_launch_dependents();
+  // 32-bit indices: the planner guarantees n*H*W*C < 2^31
   const int chunks = p.C >> 3;
-  const int64_t total = static_cast<int64_t>(p.n) * p.P * p.Q * chunks;
+  const int total = p.n * p.P * p.Q * chunks;
   const uint4* x = reinterpret_cast<const uint4*>(p.x);
   const uint4* w = reinterpret_cast<const uint4*>(p.w);
-  for (int64_t idx = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; idx < total;
-       idx += static_cast<int64_t>(gridDim.x) * blockDim.x) {
-    int64_t t = idx;
-    const int ch = static_cast<int>(t % chunks);
+  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
+    int t = idx;
+    const int ch = t % chunks;
     t /= chunks;
-    const int q = static_cast<int>(t % p.Q);
+    const int q = t % p.Q;
     t /= p.Q;
-    const int pp = static_cast<int>(t % p.P);
-    const int n = static_cast<int>(t / p.P);
+    const int pp = t % p.P;
+    const int n = t / p.P;
     float acc[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = 0.f;
@@ -175,7 +175,7 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
         const int iw = iw0 + s * p.dw;
         if (iw < 0 || iw >= p.W) continue;
         float xf[8], wf[8];
-        unpack_bf16x8(__ldg(x + ((static_cast<int64_t>(n) * p.H + ih) * p.W + iw) * chunks + ch), xf);
+        unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), xf);
         unpack_bf16x8(__ldg(w + (r * p.S + s) * chunks + ch), wf);
 #pragma unroll
         for (int i = 0; i < 8; ++i) acc[i] = fmaf(xf[i], wf[i], acc[i]);

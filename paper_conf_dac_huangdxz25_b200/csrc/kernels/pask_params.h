@@ -28,7 +28,8 @@ struct alignas(64) GemmParams {
   const void* res;     // bf16 residual, same indexing as out (nullable)
   const float* bias;   // fp32 [N] (nullable)
   float* ws_partial;   // split-K fp32 partial tiles
-  uint32_t* ws_counter;  // split-K arrival counters (self-resetting)
+  uint32_t* ws_counter;  // unused (split-K reduces on chip); kept for layout stability
+  unsigned long long* trace;  // debug: per-CTA %globaltimer phase stamps (null in production)
   int64_t ldc, off_c, stride_c;
   int32_t M, N, K, batch;
   int32_t num_kb;        // ceil(K / 64)

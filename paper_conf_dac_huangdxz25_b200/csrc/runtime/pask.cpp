@@ -30,8 +30,23 @@
 
 #define PASK_API extern "C" __attribute__((visibility("default")))
 
+// Code objects embedded by build.py (fatbins.S): the whole catalog, and one
+// SASS-only fatbin per catalog kernel.
 extern "C" const unsigned char pask_fatbin_start[];
 extern "C" const unsigned char pask_fatbin_end[];
+#define PASK_FB(k)                                    \
+  extern "C" const unsigned char pask_fb_##k##_start[]; \
+  extern "C" const unsigned char pask_fb_##k##_end[];
+PASK_FB(pask_layout)
+PASK_FB(pask_conv_igemm)
+PASK_FB(pask_conv_1x1)
+PASK_FB(pask_conv_dw)
+PASK_FB(pask_pool)
+PASK_FB(pask_pool_gavg)
+PASK_FB(pask_gemm)
+PASK_FB(pask_softmax)
+PASK_FB(pask_layernorm)
+#undef PASK_FB
 
 namespace pask {
 
@@ -67,6 +82,17 @@ struct Launch {
   std::unique_ptr<AnyParams> params;
 };
 
+struct Image {
+  const unsigned char* begin;
+  const unsigned char* end;
+};
+#define PASK_IMG(k) {pask_fb_##k##_start, pask_fb_##k##_end}
+const Image kKernelImage[PASK_NUM_KERNELS] = {
+    PASK_IMG(pask_layout),    PASK_IMG(pask_conv_igemm), PASK_IMG(pask_conv_1x1),
+    PASK_IMG(pask_conv_dw),   PASK_IMG(pask_pool),       PASK_IMG(pask_pool_gavg),
+    PASK_IMG(pask_gemm),      PASK_IMG(pask_softmax),    PASK_IMG(pask_layernorm)};
+#undef PASK_IMG
+
 bool is_gemm_kernel(int32_t k) {
   return k == PASK_K_CONV_IGEMM || k == PASK_K_CONV_1X1 || k == PASK_K_GEMM;
 }
@@ -86,7 +112,8 @@ struct Ctx {
   std::deque<int32_t> fifo;
   bool stop = false;
   std::mutex lib_mu;  // serialises library/function loads (loader vs reactive issuer)
-  CUlibrary lib = nullptr;
+  CUlibrary lib = nullptr;                     // packaging 1: the whole catalog
+  CUlibrary klib[PASK_NUM_KERNELS] = {};       // packaging 0: one code object per kernel
   std::atomic<int32_t> ready[PASK_NUM_KERNELS];
   CUfunction fn[PASK_NUM_KERNELS] = {};
   CUresult kerr[PASK_NUM_KERNELS] = {};
@@ -117,6 +144,7 @@ struct Ctx {
   bool pending = false;
   CUevent ev0 = nullptr, ev1 = nullptr;
   std::vector<CUevent> node_ev;
+  std::vector<uint64_t> node_ns;
 
   Ctx() {
     for (auto& r : ready) r.store(0);
@@ -139,22 +167,27 @@ void load_kernel(Ctx* c, int32_t k) {
   const uint64_t t0 = now_ns();
   const Driver* d = c->d;
   CUresult r = CUDA_SUCCESS;
-  if (!c->lib) {
-    const size_t bytes = static_cast<size_t>(pask_fatbin_end - pask_fatbin_start);
-    r = d->cuLibraryLoadData(&c->lib, pask_fatbin_start, nullptr, nullptr, 0, nullptr, nullptr, 0);
+  // the embedded image stays valid for the life of the process: no driver copy
+  CUlibraryOption opt[1] = {CU_LIBRARY_BINARY_IS_PRESERVED};
+  void* optv[1] = {reinterpret_cast<void*>(1)};
+  CUlibrary* lib = c->cfg.packaging == 1 ? &c->lib : &c->klib[k];
+  if (!*lib) {
+    const unsigned char* img = c->cfg.packaging == 1 ? pask_fatbin_start : kKernelImage[k].begin;
+    const unsigned char* end = c->cfg.packaging == 1 ? pask_fatbin_end : kKernelImage[k].end;
+    r = d->cuLibraryLoadData(lib, img, nullptr, nullptr, 0, opt, optv, 1);
     c->k_lib_ns[k] = now_ns() - t0;
     if (r == CUDA_SUCCESS) {
       c->code_objects.fetch_add(1);
-      c->code_bytes.fetch_add(bytes);
+      c->code_bytes.fetch_add(static_cast<uint64_t>(end - img));
     }
   }
   CUkernel kern = nullptr;
   CUfunction f = nullptr;
-  if (r == CUDA_SUCCESS) r = d->cuLibraryGetKernel(&kern, c->lib, catalog(k).name);
+  if (r == CUDA_SUCCESS) r = d->cuLibraryGetKernel(&kern, *lib, catalog(k).name);
   if (r == CUDA_SUCCESS) r = d->cuKernelGetFunction(&f, kern);
   if (r == CUDA_SUCCESS) r = d->cuFuncLoad(f);
   if (r == CUDA_SUCCESS && is_gemm_kernel(k))
-    r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 210 * 1024);  // >= gemm_tiling max (200 KB ring + barriers + align)
+    r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, static_cast<int>(kMaxDynSmem));
   if (r == CUDA_SUCCESS && is_gemm_kernel(k))  // one fixed L1/smem split: no per-launch reconfiguration
     r = d->cuFuncSetAttribute(f, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100);
   c->fn[k] = f;
@@ -356,6 +389,11 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
                          static_cast<uint64_t>(batch), static_cast<uint64_t>(nd.ldb) * 2,
                          static_cast<uint64_t>(nd.stride_b) * 2, 64, 64, err);
         if (rc) return rc;
+      }
+      {  // debug-only phase trace (PASK_TRACE_NODE=i PASK_TRACE_PTR=<device address>)
+        const char* tn = getenv("PASK_TRACE_NODE");
+        const char* tp = getenv("PASK_TRACE_PTR");
+        if (tn && tp && atoi(tn) == i) q.trace = reinterpret_cast<unsigned long long*>(strtoull(tp, nullptr, 0));
       }
       L.block[0] = kGemmThreads;
       L.grid[0] = static_cast<unsigned>(t.m_tiles);
@@ -644,10 +682,13 @@ PASK_API int pask_sync(pask_ctx* c) {
     c->st.gpu_span_ns = static_cast<uint64_t>(ms * 1e6);
   if (c->cfg.instrument) {
     uint64_t busy = 0;
+    c->node_ns.assign(c->node_ev.size() / 2, 0);
     for (size_t i = 0; i + 1 < c->node_ev.size(); i += 2) {
       float e = 0.f;
-      if (d->cuEventElapsedTime(&e, c->node_ev[i], c->node_ev[i + 1]) == CUDA_SUCCESS)
-        busy += static_cast<uint64_t>(e * 1e6);
+      if (d->cuEventElapsedTime(&e, c->node_ev[i], c->node_ev[i + 1]) == CUDA_SUCCESS) {
+        c->node_ns[i / 2] = static_cast<uint64_t>(e * 1e6);
+        busy += c->node_ns[i / 2];
+      }
     }
     c->st.gpu_busy_ns = busy;
   }
@@ -713,6 +754,15 @@ PASK_API int pask_kernel_timeline(const pask_ctx* c, int32_t k, uint64_t* load_n
   return PASK_OK;
 }
 
+PASK_API int pask_node_times(const pask_ctx* c, uint64_t* ns_out, int32_t n) {
+  t_err.clear();
+  if (!c || !ns_out) return set_err(PASK_EINVAL, "null argument");
+  if (!c->cfg.instrument) return set_err(PASK_ESTATE, "context not created with instrument = 1");
+  if (n != static_cast<int32_t>(c->node_ns.size())) return set_err(PASK_EINVAL, "n_nodes mismatch (sync first)");
+  for (int32_t i = 0; i < n; ++i) ns_out[i] = c->node_ns[i];
+  return PASK_OK;
+}
+
 PASK_API int pask_destroy(pask_ctx* c) {
   t_err.clear();
   if (!c) return PASK_OK;
@@ -729,6 +779,8 @@ PASK_API int pask_destroy(pask_ctx* c) {
   if (c->ev0) d->cuEventDestroy(c->ev0);
   if (c->ev1) d->cuEventDestroy(c->ev1);
   if (c->lib) d->cuLibraryUnload(c->lib);
+  for (CUlibrary l : c->klib)
+    if (l) d->cuLibraryUnload(l);
   delete c;
   return PASK_OK;
 }

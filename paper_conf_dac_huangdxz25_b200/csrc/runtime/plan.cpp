@@ -50,6 +50,7 @@ pask_config default_config() {
   c.proactive = 1;
   c.pdl = 1;
   c.instrument = 0;
+  c.packaging = 0;
   return c;
 }
 
@@ -62,6 +63,7 @@ bool is_applicable(int32_t id, const Problem& p, std::string* why) {
   switch (id) {
     case PASK_K_LAYOUT:
       if (p.op != OC_LAYOUT) return fail("not a layout op");
+      if (static_cast<int64_t>(p.n) * p.h * p.w * std::max(p.c, p.k) >= (1ll << 31)) return fail("tensor too large for 32-bit indexing");
       if (p.k % 8 != 0) return fail("padded channels % 8 != 0");
       if (p.c > p.k) return fail("input channels exceed padded channels");
       return true;
@@ -83,6 +85,7 @@ bool is_applicable(int32_t id, const Problem& p, std::string* why) {
       return true;
     case PASK_K_CONV_DW:
       if (p.op != OC_DWCONV) return fail("not a depthwise conv");
+      if (static_cast<int64_t>(p.n) * p.h * p.w * p.c >= (1ll << 31)) return fail("tensor too large for 32-bit indexing");
       if (p.c % 8 != 0) return fail("C % 8 != 0");
       if (p.r < 1 || p.r > 15 || p.s < 1 || p.s > 15) return fail("filter size outside [1,15]");
       if (p.stride_h < 1 || p.stride_h > 8 || p.stride_w < 1 || p.stride_w > 8) return fail("stride outside [1,8]");
@@ -91,6 +94,7 @@ bool is_applicable(int32_t id, const Problem& p, std::string* why) {
       return true;
     case PASK_K_POOL:
       if (p.op != OC_POOL) return fail("not a pool");
+      if (static_cast<int64_t>(p.n) * p.h * p.w * p.c >= (1ll << 31)) return fail("tensor too large for 32-bit indexing");
       if (p.c % 8 != 0) return fail("C % 8 != 0");
       if (static_cast<int64_t>(p.r) * p.s > 1024) return fail("window larger than 1024 taps");
       if (p.stride_h < 1 || p.stride_w < 1) return fail("stride < 1");
@@ -384,15 +388,16 @@ GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b
   t.rows_per = 128 / splits;
   const int32_t kb_per = (t.num_kb + splits - 1) / splits;
   const uint32_t stage_bytes = 16384u + static_cast<uint32_t>(t.bn) * 128u;
-  int32_t stages = static_cast<int32_t>((160u * 1024u) / stage_bytes);
+  const uint32_t recv = splits > 1 ? ((128u * (t.bn + 4) * 4 + 1023u) & ~1023u) : 0u;
+  const uint32_t ro = c_tma ? ((128u * t.bn * 2 + 1023u) & ~1023u) : 0u;
+  const uint32_t fixed = recv + ro + 1024u /*bias*/ + 256u /*barriers*/ + 1024u /*align slack*/;
+  const uint32_t budget = kMaxDynSmem - fixed;  // ring gets what is left, at most 8 stages
+  int32_t stages = static_cast<int32_t>(budget / stage_bytes);
   stages = std::min(stages, 8);
   stages = std::min(stages, std::max(2, kb_per));
   t.stages = std::max(2, stages);
-  const uint32_t ring = t.stages * stage_bytes;
-  const uint32_t stage32 = splits > 1 ? 128u * (t.bn + 4) * 4 : 0u;
-  const uint32_t reg0 = (std::max(ring, stage32) + 1023u) & ~1023u;
-  const uint32_t ro = c_tma ? ((128u * t.bn * 2 + 1023u) & ~1023u) : 0u;
-  t.smem_bytes = reg0 + ro + 1024u /*bias*/ + (2 * t.stages + 3) * 8u + 1024u /*align slack*/;
+  const uint32_t ring = (t.stages * stage_bytes + 1023u) & ~1023u;
+  t.smem_bytes = ring + fixed;
   uint32_t cols = 32;
   while (cols < static_cast<uint32_t>(t.bn)) cols <<= 1;
   t.tmem_cols = cols;

@@ -58,6 +58,8 @@ struct GemmTiling {
   int32_t bn, m_tiles, n_tiles, num_kb, splits, rows_per, stages;
   uint32_t smem_bytes, tmem_cols;
 };
+// Dynamic shared memory the contraction kernels may request (attribute set at load).
+constexpr uint32_t kMaxDynSmem = 220u * 1024u;
 // c_tma: output / residual go through smem staging + TMA (changes the smem size)
 GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma);
 

@@ -55,7 +55,8 @@ class Graph(C.Structure):
 
 class Config(C.Structure):
     _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
-                ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32)]
+                ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
+                ("packaging", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -78,7 +79,7 @@ class Stats(C.Structure):
 EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "pask_load_model",
            "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
            "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name",
-           "pask_kernel_timeline"]
+           "pask_kernel_timeline", "pask_node_times"]
 
 _lib = None
 
@@ -108,6 +109,7 @@ def lib():
         "pask_destroy": (C.c_int, [P]),
         "pask_kernel_timeline": (C.c_int, [P, C.c_int32, C.POINTER(C.c_uint64),
                                            C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
+        "pask_node_times": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int32]),
         "pask_last_error": (C.c_char_p, []),
         "pask_num_kernels": (C.c_int32, []),
         "pask_kernel_name": (C.c_char_p, [C.c_int32]),
@@ -136,8 +138,8 @@ def kernel_name(k):
     return lib().pask_kernel_name(k).decode()
 
 
-def config(reuse=1, search=0, milestone=0, proactive=1, pdl=1, instrument=0):
-    return Config(reuse, search, milestone, proactive, pdl, instrument)
+def config(reuse=1, search=0, milestone=0, proactive=1, pdl=1, instrument=0, packaging=0):
+    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging)
 
 
 def plan(graph: Graph, cfg: Config | None = None):
@@ -199,6 +201,12 @@ class Context:
         a, b, c = C.c_uint64(), C.c_uint64(), C.c_uint64()
         _check(lib().pask_kernel_timeline(self.h, k, C.byref(a), C.byref(b), C.byref(c)))
         return a.value, b.value, c.value
+
+    def node_times(self):
+        """Per-node GPU ns of the last instrumented inference (cfg.instrument = 1)."""
+        arr = (C.c_uint64 * max(self.n_nodes, 1))()
+        _check(lib().pask_node_times(self.h, arr, self.n_nodes))
+        return list(arr[:self.n_nodes])
 
     def close(self):
         if self.h:

@@ -27,10 +27,38 @@ def test_model_layers_teacher_forced(name):
     assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
     st = ctx.stats()
     assert st["kernels_loaded"] == len(o["loaded"])
-    assert st["code_objects_loaded"] == 1
+    assert st["code_objects_loaded"] == len(o["loaded"])   # packaging 0: one object per kernel
     loaded = {k for k in range(P.NUM_KERNELS) if ctx.kernel_is_loaded(k)}
     assert loaded == set(o["loaded"])
     assert len(loaded) <= 8
+    ctx.close()
+
+
+@pytest.mark.parametrize("packaging", [0, 1])
+@pytest.mark.parametrize("cfg", ["reactive", "pask_i", "pask_r", "no_pdl"])
+def test_schemes_same_outputs(cfg, packaging):
+    """Every scheme of PAPER.md:174-186 (reactive loading, PaSK-I = no reuse,
+    PaSK-R = naive search) and both code-object packagings produce outputs
+    within tolerance; plans match the plan oracle for the same config."""
+    spec, x = build_model("resnet50")
+    kw = dict(packaging=packaging)
+    if cfg == "reactive":
+        kw.update(proactive=0)
+    elif cfg == "pask_i":
+        kw.update(reuse=0)
+    elif cfg == "pask_r":
+        kw.update(search=1)
+    else:
+        kw.update(pdl=0)
+    dm, ctx, plan = run_model(spec, x, cfg=P.config(**kw))
+    errs = teacher_forced_errors(dm, spec, x)
+    assert max(e for _, _, e in errs) <= TOL
+    o = OP.execution_plan(OP.problems_from_spec(spec), reuse=bool(kw.get("reuse", 1)),
+                          search="naive" if kw.get("search") else "categorical")
+    assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
+    st = ctx.stats()
+    assert st["kernels_loaded"] == len(o["loaded"])
+    assert st["code_objects_loaded"] == (1 if packaging == 1 else len(o["loaded"]))
     ctx.close()
 
 
