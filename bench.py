@@ -248,12 +248,14 @@ def main():
     barrier()
     torch.cuda.synchronize()
     t0 = time.perf_counter_ns()
-    plan = ctx.load_model(dm.graph)
+    ctx.load_model(dm.graph, plan=False)
     ctx.infer(sp)
     ctx.sync()
     t1 = time.perf_counter_ns()
-    cold_ms = (t1 - t0) / 1e6
+    plan = ctx.bindings()
     cold_stats = ctx.stats()
+    cold_ms = cold_stats["cold_wall_ns"] / 1e6      # library clock: load_model entry -> sync return
+    cold_py_ms = (t1 - t0) / 1e6                    # the same window seen from Python
     timeline = {}
     for k in range(P.NUM_KERNELS):
         ld, rd, lb = ctx.kernel_timeline(k)
@@ -395,6 +397,7 @@ def main():
                    "l2": "warm (no flush)" if args.no_flush else
                          "flushed (256 MiB memset) before every timed inference"},
         "cold_ms": round(cold_max, 3),
+        "cold_ms_python_clock": round(cold_py_ms, 3),
         "hot_ms": round(hot_max, 4),
         "cold_over_hot": round(cold_max / hot_max, 3),
         "hot_l2_warm_ms": round(warm_max, 4),

@@ -170,12 +170,22 @@ typedef struct {
   int32_t reuse;      /* 1 = Algorithm 1 reuse (PaSK); 0 = always load s* (PaSK-I / Baseline) */
   int32_t search;     /* 0 = categorical MRU lists; 1 = naive scan (PaSK-R, :186) */
   int32_t milestone;  /* m of PAPER.md:97; layers 1..m load s* unconditionally (default 0)    */
-  int32_t proactive;  /* 1 = loader thread; 0 = reactive load at first launch   */
+  int32_t proactive;  /* 1 = loader thread started at parse time;
+                         2 = the caller thread uploads every planned kernel inside
+                             pask_load_model, right after planning (a hot core; fastest
+                             measured on B200, D5);
+                         0 = reactive: each kernel loaded at its first launch (A1 baseline) */
   int32_t pdl;        /* 1 = programmatic dependent launch between consecutive kernels        */
   int32_t instrument; /* 1 = per-node CUDA events for gpu_busy_ns (perturbs timing)           */
   int32_t packaging;  /* 0 = one code object per catalog kernel (default: a load costs ~0.9 us
                          per KB of image, so only the bound kernels' code is parsed);
                          1 = the whole catalog as one code object                            */
+  int32_t interleave; /* 0 = load-first (default): the first inference launches once every
+                         planned kernel is uploaded -- on this driver a code upload waits for
+                         all running GPU work, so
+                         uploads are done while the GPU is idle anyway;
+                         1 = Fig. 5 interleaving: launch each layer as soon as its kernel is
+                         ready (the loader yields to the issuer)                             */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;
@@ -206,14 +216,19 @@ typedef struct {
   uint64_t cold_wall_ns;       /* pask_load_model entry -> first inference done   */
   uint64_t infer_count;
   uint64_t launches;           /* kernel launches issued so far                   */
+  uint64_t load_done_ns;       /* cold timeline, ns after pask_load_model entry:  */
+  uint64_t infer_entry_ns;     /*   last planned kernel uploaded, first pask_infer */
+  uint64_t first_launch_ns;    /*   entry, its first and last launch              */
+  uint64_t last_launch_ns;
 } pask_stats_t;
 
 /* Library version (PASK_VERSION). */
 int pask_version(void);
 
 /* Create a context bound to the device's primary context (the one PyTorch
- * uses) and start the (idle) loader thread.  cfg may be NULL for defaults
- * {reuse 1, search 0, milestone 0, proactive 1, pdl 1, instrument 0}. */
+ * uses) and start the (idle) helper/loader thread.  cfg may be NULL for
+ * defaults {reuse 1, search 0, milestone 0, proactive 2, pdl 1, instrument 0,
+ * packaging 0, interleave 0}. */
 int pask_create(pask_ctx **ctx, int device, const pask_config *cfg);
 
 /* Host-only planning (no GPU needed): validate g, extract problems p_i, apply
@@ -228,10 +243,15 @@ int pask_plan(const pask_graph *g, const pask_config *cfg, pask_binding *plan_ou
  * tile counters); host-only. */
 int pask_workspace_bytes(const pask_graph *g, uint64_t *bytes);
 
-/* Plan g (synchronously), hand the bound kernels to the loader thread in
- * first-use order (asynchronously) and encode per-node launch parameters while
- * loading proceeds.  plan_out may be NULL.  The graph arrays are copied; the
- * device buffers they point to are not. */
+/* Plan g (Algorithm 1), then load the bound kernels in first-use order while
+ * the per-node launch parameters are encoded concurrently:
+ *   proactive 2 (default): the caller thread uploads, the helper thread encodes,
+ *                          and the call returns with every kernel resident;
+ *   proactive 1: the loader thread uploads asynchronously, the
+ *                caller encodes and returns; pask_infer waits for / steals loads;
+ *   proactive 0: nothing is loaded here (reactive baseline).
+ * plan_out may be NULL.  The graph arrays are copied; the device buffers they
+ * point to are not. */
 int pask_load_model(pask_ctx *ctx, const pask_graph *g, pask_binding *plan_out);
 
 /* Issue one inference on cuda_stream (a CUstream / cudaStream_t; NULL = legacy

@@ -156,6 +156,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const uint32_t recv = smem_base + ring_bytes;  // slot s: rows [s*rows_per, (s+1)*rows_per)
 
   const bool gather = kAllowGather && (p.a_mode == A_GATHER);
+  const bool im2col = kAllowGather && (p.a_mode == A_IM2COL);
   const int mt = blockIdx.x, nt = blockIdx.y;
   const int b = blockIdx.z / splits;
   const int split = blockIdx.z - b * splits;
@@ -212,6 +213,22 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           tma_load_3d(ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), &p.tmap_r, res_bar,
                       n0 + j * box_cols, m0 + r0, b);
       }
+      // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
+      int iw = 0, ih = 0, in = 0, cc = 0, tr = 0, ts = 0;
+      const int cpt = p.C >> 6;  // 64-channel chunks per filter tap
+      if (kAllowGather && im2col) {
+        const int pq = p.P * p.Q;
+        in = m0 / pq;
+        const int rem = m0 - in * pq;
+        const int pp = rem / p.Q;
+        const int qq = rem - pp * p.Q;
+        iw = qq * p.sw - p.pw;
+        ih = pp * p.sh - p.ph;
+        const int tap = kb_begin / cpt;
+        cc = kb_begin - tap * cpt;
+        tr = tap / p.S;
+        ts = tap - tr * p.S;
+      }
       int s = 0;
       uint32_t ph = 0;
       for (int i = 0; i < nk; ++i) {
@@ -220,7 +237,19 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const uint32_t sb = sa + kABytes;
         const int kb = kb_begin + i;
         mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
-        if (!gather) tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
+        if (kAllowGather && im2col) {
+          tma_load_im2col_4d(sa, &p.tmap_a, full0 + 8 * s, cc * 64, iw, ih, in,
+                             static_cast<uint16_t>(ts * p.dw), static_cast<uint16_t>(tr * p.dh));
+          if (++cc == cpt) {
+            cc = 0;
+            if (++ts == p.S) {
+              ts = 0;
+              ++tr;
+            }
+          }
+        } else if (!gather) {
+          tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
+        }
         if (p.b_major == 0) {
           tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
         } else {

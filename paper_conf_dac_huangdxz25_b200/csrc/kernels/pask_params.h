@@ -15,11 +15,13 @@ constexpr int kGemmThreads = 192;  // warps 0-3 gather/epilogue, 4 TMA, 5 TMEM+M
 // A-operand source of the contraction kernel.
 enum AMode : int32_t {
   A_TMA = 0,     // A is a plain K-major matrix: TMA tiled load (GEMM, 1x1 s1 p0 conv)
-  A_GATHER = 1,  // implicit im2col: cp.async gather with runtime pad/stride/dilation
+  A_GATHER = 1,  // implicit im2col: cp.async gather with runtime pad/stride/dilation (any C % 8)
+  A_IM2COL = 2,  // implicit im2col by TMA im2col mode (C % 64 == 0): one load per (tap, 64 ch)
 };
 
 struct alignas(64) GemmParams {
   CUtensorMap tmap_a;  // A_TMA: 3-D {K, M, batch}, box {64, 128, 1}, SWIZZLE_128B
+                       // A_IM2COL: 4-D im2col {C, W, H, N}, 64 ch x 128 px, corners -pad / pad-(R-1)dil
   CUtensorMap tmap_b;  // K-major: {K, N, batch} box {64, BN, 1}; MN-major: {N, K, batch} box {64, 64, 1}
   CUtensorMap tmap_c;  // c_tma: output {N, M, batch} (ldc), box {64, rows_per, 1}, SWIZZLE_128B
   CUtensorMap tmap_r;  // c_tma && res: residual, same geometry as tmap_c with box {64, 128, 1}

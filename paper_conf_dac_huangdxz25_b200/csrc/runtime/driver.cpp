@@ -52,6 +52,7 @@ void resolve() {
   PASK_RESOLVE(cuFuncSetAttribute)
   PASK_RESOLVE(cuLaunchKernelEx)
   PASK_RESOLVE(cuTensorMapEncodeTiled)
+  PASK_RESOLVE(cuTensorMapEncodeIm2col)
   PASK_RESOLVE(cuEventCreate)
   PASK_RESOLVE(cuEventDestroy)
   PASK_RESOLVE(cuEventRecord)

@@ -26,6 +26,7 @@ struct Driver {
   PASK_DRV_FN(cuFuncSetAttribute)
   PASK_DRV_FN(cuLaunchKernelEx)
   PASK_DRV_FN(cuTensorMapEncodeTiled)
+  PASK_DRV_FN(cuTensorMapEncodeIm2col)
   PASK_DRV_FN(cuEventCreate)
   PASK_DRV_FN(cuEventDestroy)
   PASK_DRV_FN(cuEventRecord)

@@ -122,6 +122,17 @@ struct Ctx {
   std::atomic<int32_t> code_objects{0};
   std::atomic<uint64_t> code_bytes{0};
   std::atomic<int32_t> kernels_loaded{0};
+  // Issue priority: a code-object load holds the driver for 30-90 us and stalls
+  // concurrent cuLaunchKernelEx calls (measured: 32 us per launch during a
+  // load burst vs 2.4 us).  The loader therefore starts a load only while the
+  // issuer is not issuing (blocked on a missing kernel, or between inferences);
+  // the GPU keeps executing the already-queued layers meanwhile.
+  std::atomic<int32_t> issuing{0};
+  // proactive = 2: the helper thread encodes launch parameters (job kEncodeJob)
+  // while the caller thread uploads the planned kernels
+  std::atomic<int32_t> encode_state{0};  // 0 idle, 1 queued/running, 2 done
+  int encode_rc = 0;
+  std::string encode_err;
   uint64_t k_load_ns[PASK_NUM_KERNELS] = {};   // per-kernel cold timeline
   uint64_t k_ready_at[PASK_NUM_KERNELS] = {};  // absolute steady-clock ns
   uint64_t k_lib_ns[PASK_NUM_KERNELS] = {};
@@ -152,6 +163,9 @@ struct Ctx {
 };
 
 namespace {
+
+constexpr int32_t kEncodeJob = -1;
+int encode_all(Ctx* c, std::string* err);
 
 std::string cu_err(const Driver* d, CUresult r, const char* what) {
   const char* name = nullptr;
@@ -200,19 +214,45 @@ void load_kernel(Ctx* c, int32_t k) {
   c->ready[k].store(r == CUDA_SUCCESS ? 1 : -1, std::memory_order_release);
 }
 
+// The loader polls for work (keeping its core awake) for a bounded window after
+// each wake-up -- a load started on a just-woken, down-clocked core measured up
+// to 7x slower -- then sleeps on the condition variable.
 void loader_main(Ctx* c) {
   pthread_setname_np(pthread_self(), "pask-loader");
   c->d->cuCtxSetCurrent(c->cuctx);
+  constexpr uint64_t kSpinNs = 20ull * 1000 * 1000;  // 20 ms
+  uint64_t spin_until = now_ns() + kSpinNs;
   for (;;) {
-    int32_t k;
-    {
-      std::unique_lock<std::mutex> lk(c->mu);
-      c->cv.wait(lk, [&] { return c->stop || !c->fifo.empty(); });
-      if (c->stop && c->fifo.empty()) return;
-      k = c->fifo.front();
-      c->fifo.pop_front();
+    int32_t k = 0;
+    bool got = false;
+    while (!got) {
+      {
+        std::unique_lock<std::mutex> lk(c->mu);
+        if (c->stop && c->fifo.empty()) return;
+        if (!c->fifo.empty()) {
+          k = c->fifo.front();
+          c->fifo.pop_front();
+          got = true;
+          break;
+        }
+        if (now_ns() > spin_until) {
+          c->cv.wait(lk, [&] { return c->stop || !c->fifo.empty(); });
+          spin_until = now_ns() + kSpinNs;
+          continue;
+        }
+      }
+      for (int i = 0; i < 64; ++i) _mm_pause();
     }
+    if (k == kEncodeJob) {
+      c->encode_rc = encode_all(c, &c->encode_err);
+      c->encode_state.store(2, std::memory_order_release);
+      spin_until = now_ns() + kSpinNs;
+      continue;
+    }
+    if (c->cfg.interleave)
+      while (c->issuing.load(std::memory_order_acquire) && !c->stop) _mm_pause();
     load_kernel(c, k);
+    spin_until = now_ns() + kSpinNs;
   }
 }
 
@@ -358,7 +398,13 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
       if (p.op == OC_CONV) {
         const bool plain = (p.r == 1 && p.s == 1 && p.stride_h == 1 && p.stride_w == 1 && p.pad_h == 0 &&
                             p.pad_w == 0);
-        q.a_mode = (L.kernel == PASK_K_CONV_1X1 || plain) ? A_TMA : A_GATHER;
+        // TMA im2col needs whole 64-channel chunks per tap and its corner ranges
+        const int lw = -p.pad_w, lh = -p.pad_h;
+        const int uw = p.pad_w - (p.s - 1) * p.dil_w, uh = p.pad_h - (p.r - 1) * p.dil_h;
+        const bool im2col_ok = (p.c % 64 == 0) && lw >= -128 && lh >= -128 && uw >= -128 && uh >= -128 &&
+                               uw <= 127 && uh <= 127 && (p.s - 1) * p.dil_w < 65536 && (p.r - 1) * p.dil_h < 65536 &&
+                               !getenv("PASK_NO_IM2COL");
+        q.a_mode = (L.kernel == PASK_K_CONV_1X1 || plain) ? A_TMA : (im2col_ok ? A_IM2COL : A_GATHER);
         q.x = x.dptr;
         q.H = p.h; q.W = p.w; q.C = p.c; q.P = p.p; q.Q = p.q; q.R = p.r; q.S = p.s;
         q.sh = p.stride_h; q.sw = p.stride_w; q.ph = p.pad_h; q.pw = p.pad_w; q.dh = p.dil_h; q.dw = p.dil_w;
@@ -366,6 +412,22 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
           rc = encode_3d(c, &q.tmap_a, x.dptr, static_cast<uint64_t>(K), static_cast<uint64_t>(M), 1,
                          static_cast<uint64_t>(p.c) * 2, 0, 64, 128, err);
           if (rc) return rc;
+        } else if (q.a_mode == A_IM2COL) {
+          cuuint64_t dims[4] = {static_cast<cuuint64_t>(p.c), static_cast<cuuint64_t>(p.w),
+                                static_cast<cuuint64_t>(p.h), static_cast<cuuint64_t>(p.n)};
+          cuuint64_t strides[3] = {static_cast<cuuint64_t>(p.c) * 2, static_cast<cuuint64_t>(p.w) * p.c * 2,
+                                   static_cast<cuuint64_t>(p.h) * p.w * p.c * 2};
+          int lower[2] = {lw, lh}, upper[2] = {uw, uh};  // {W, H} (innermost spatial first)
+          cuuint32_t es[4] = {1, static_cast<cuuint32_t>(p.stride_w), static_cast<cuuint32_t>(p.stride_h), 1};
+          CUresult r = c->d->cuTensorMapEncodeIm2col(&q.tmap_a, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, x.dptr, dims,
+                                                     strides, lower, upper, 64, 128, es,
+                                                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                                                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+          if (r != CUDA_SUCCESS) {
+            *err = cu_err(c->d, r, "cuTensorMapEncodeIm2col");
+            return PASK_ECUDA;
+          }
         }
         // weights KRSC = [N][K] K-major
         rc = encode_3d(c, &q.tmap_b, nd.w, static_cast<uint64_t>(K), static_cast<uint64_t>(N), 1,
@@ -408,6 +470,14 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
   return PASK_EINVAL;
 }
 
+int encode_all(Ctx* c, std::string* err) {
+  for (int32_t i = 0; i < static_cast<int32_t>(c->nodes.size()); ++i) {
+    int rc = lower_node(c, i, err);
+    if (rc) return rc;
+  }
+  return PASK_OK;
+}
+
 int plan_graph(const pask_graph* g, const pask_config& cfg, std::vector<Problem>* probs, PlanResult* plan) {
   std::string err;
   int rc = extract_problems(g, probs, &err);
@@ -422,21 +492,38 @@ int plan_graph(const pask_graph* g, const pask_config& cfg, std::vector<Problem>
   return PASK_OK;
 }
 
+// Wait until kernel k is loaded.  A blocked issuer does not idle: it pops the
+// next queued load (first-use order) and performs it itself -- its core is
+// already running, while the loader thread may be waking on a cold core.
 int wait_kernel(Ctx* c, int32_t k) {
   int32_t s = c->ready[k].load(std::memory_order_acquire);
   if (s == 0) {
     const uint64_t t0 = now_ns();
+    c->issuing.store(0, std::memory_order_release);  // blocked: the loader may take the driver
     if (!c->cfg.proactive) {
       load_kernel(c, k);  // reactive: load at launch, on the issue thread (A1 baseline)
     } else {
-      if (!c->requested[k]) {  // not planned for loading (e.g. rebinding) -> queue it now
-        std::lock_guard<std::mutex> lk(c->mu);
-        c->requested[k] = true;
-        c->fifo.push_back(k);
-        c->cv.notify_one();
+      for (;;) {
+        if ((s = c->ready[k].load(std::memory_order_acquire)) != 0) break;
+        int32_t next = -1;
+        {
+          std::lock_guard<std::mutex> lk(c->mu);
+          if (!c->requested[k]) {  // not planned for loading (e.g. rebinding) -> queue it now
+            c->requested[k] = true;
+            c->fifo.push_back(k);
+          }
+          if (!c->fifo.empty()) {
+            next = c->fifo.front();
+            c->fifo.pop_front();
+          }
+        }
+        if (next >= 0)
+          load_kernel(c, next);  // work stealing; lib_mu keeps loads serialised
+        else
+          _mm_pause();  // the loader thread holds the last pending load
       }
-      while ((s = c->ready[k].load(std::memory_order_acquire)) == 0) _mm_pause();
     }
+    c->issuing.store(1, std::memory_order_release);
     c->st.load_exposed_ns += now_ns() - t0;
     s = c->ready[k].load(std::memory_order_acquire);
   }
@@ -557,19 +644,7 @@ PASK_API int pask_load_model(pask_ctx* c, const pask_graph* g, pask_binding* pla
   int rc = plan_graph(g, c->cfg, &c->probs, &c->plan);
   if (rc) return rc;
   const uint64_t t_plan = now_ns();
-  // ---- proactive loading: hand the bound kernels to the loader, first-use order
-  if (c->cfg.proactive) {
-    std::lock_guard<std::mutex> lk(c->mu);
-    for (const pask_binding& b : c->plan.bindings) {
-      const int32_t k = b.bound_kernel;
-      if (!c->requested[k]) {
-        c->requested[k] = true;
-        c->fifo.push_back(k);
-      }
-    }
-    c->cv.notify_one();
-  }
-  // ---- copy the graph and lower every node while loading proceeds
+  // ---- copy the graph (the library keeps its own arrays)
   c->tensors.assign(g->tensors, g->tensors + g->n_tensors);
   c->nodes.assign(g->nodes, g->nodes + g->n_nodes);
   c->inputs.assign(g->inputs, g->inputs + g->n_inputs);
@@ -583,8 +658,45 @@ PASK_API int pask_load_model(pask_ctx* c, const pask_graph* g, pask_binding* pla
   c->launches.clear();
   c->launches.resize(g->n_nodes);
   std::string err;
-  for (int32_t i = 0; i < g->n_nodes; ++i) {
-    rc = lower_node(c, i, &err);
+  uint64_t t_loads = 0;
+  if (c->cfg.proactive == 2) {
+    // the caller thread uploads the planned kernels in first-use order while
+    // the helper thread encodes the per-node launch parameters
+    c->encode_state.store(1, std::memory_order_release);
+    {
+      std::lock_guard<std::mutex> lk(c->mu);
+      c->fifo.push_back(kEncodeJob);
+      c->cv.notify_one();
+    }
+    for (int32_t k : c->plan.loaded) {
+      {
+        std::lock_guard<std::mutex> lk(c->mu);
+        c->requested[k] = true;
+      }
+      load_kernel(c, k);
+    }
+    t_loads = now_ns();
+    while (c->encode_state.load(std::memory_order_acquire) != 2) _mm_pause();
+    c->encode_state.store(0, std::memory_order_release);
+    if (c->encode_rc) return set_err(c->encode_rc, c->encode_err);
+    for (int32_t k : c->plan.loaded)
+      if (c->ready[k].load(std::memory_order_acquire) < 0)
+        return set_err(PASK_ECUDA, cu_err(c->d, c->kerr[k], (std::string("loading ") + catalog(k).name).c_str()));
+  } else {
+    // ---- proactive loading: hand the bound kernels to the loader, first-use order
+    if (c->cfg.proactive) {
+      std::lock_guard<std::mutex> lk(c->mu);
+      for (const pask_binding& b : c->plan.bindings) {
+        const int32_t k = b.bound_kernel;
+        if (!c->requested[k]) {
+          c->requested[k] = true;
+          c->fifo.push_back(k);
+        }
+      }
+      c->cv.notify_one();
+    }
+    // ---- lower every node while loading proceeds
+    rc = encode_all(c, &err);
     if (rc) return set_err(rc, err);
   }
   if (c->cfg.instrument) {
@@ -602,6 +714,7 @@ PASK_API int pask_load_model(pask_ctx* c, const pask_graph* g, pask_binding* pla
   c->st.lookups = c->plan.lookups;
   c->st.plan_ns = t_plan - c->t_entry;
   c->st.encode_ns = t_enc - t_plan;
+  c->st.load_done_ns = t_loads ? t_loads - c->t_entry : 0;
   if (plan_out) memcpy(plan_out, c->plan.bindings.data(), c->plan.bindings.size() * sizeof(pask_binding));
   c->have_model = true;
   c->first_done = false;
@@ -613,6 +726,8 @@ PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, 
   if (!c) return set_err(PASK_EINVAL, "null ctx");
   if (!c->have_model) return set_err(PASK_ESTATE, "pask_infer before pask_load_model");
   int rc;
+  const bool first = c->st.infer_count == 0;
+  if (first) c->st.infer_entry_ns = now_ns() - c->t_entry;
   for (size_t i = 0; inputs && i < c->inputs.size(); ++i)
     if (inputs[i] && (rc = rebind(c, c->inputs[i], inputs[i]))) return rc;
   for (size_t i = 0; outputs && i < c->outputs.size(); ++i)
@@ -620,6 +735,18 @@ PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, 
   const Driver* d = c->d;
   CUstream s = static_cast<CUstream>(stream);
   CUlaunchAttribute attr[2];
+  if (c->cfg.proactive && !c->cfg.interleave) {
+    // load-first: every planned kernel uploaded before the first launch (uploads
+    // wait for running GPU work, so interleaving them with launches only
+    // serialises each upload behind the layers already queued)
+    for (int32_t k : c->plan.loaded)
+      if ((rc = wait_kernel(c, k))) return rc;
+  }
+  c->issuing.store(1, std::memory_order_release);
+  struct Idle {  // the loader may run again once this inference is issued (or fails)
+    std::atomic<int32_t>& f;
+    ~Idle() { f.store(0, std::memory_order_release); }
+  } idle{c->issuing};
   for (size_t i = 0; i < c->launches.size(); ++i) {
     Launch& L = c->launches[i];
     if ((rc = wait_kernel(c, L.kernel))) return rc;
@@ -658,6 +785,11 @@ PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, 
                                                catalog(L.kernel).name + ")").c_str()));
     if (c->cfg.instrument) d->cuEventRecord(c->node_ev[2 * i + 1], s);
     c->st.launches++;
+    if (first && i == 0) c->st.first_launch_ns = now_ns() - c->t_entry;
+  }
+  if (first) {
+    c->st.last_launch_ns = now_ns() - c->t_entry;
+    if (!c->st.load_done_ns) c->st.load_done_ns = c->st.first_launch_ns;
   }
   d->cuEventRecord(c->ev1, s);
   c->st.infer_count++;

@@ -47,10 +47,11 @@ pask_config default_config() {
   c.reuse = 1;
   c.search = 0;
   c.milestone = 0;
-  c.proactive = 1;
+  c.proactive = 2;
   c.pdl = 1;
   c.instrument = 0;
   c.packaging = 0;
+  c.interleave = 0;
   return c;
 }
 

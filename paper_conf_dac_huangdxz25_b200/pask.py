@@ -56,7 +56,7 @@ class Graph(C.Structure):
 class Config(C.Structure):
     _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
                 ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
-                ("packaging", C.c_int32)]
+                ("packaging", C.c_int32), ("interleave", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -70,7 +70,9 @@ class Stats(C.Structure):
                 ("lookups", C.c_int32), ("code_bytes_loaded", C.c_uint64), ("plan_ns", C.c_uint64),
                 ("load_ns", C.c_uint64), ("load_exposed_ns", C.c_uint64), ("issue_ns", C.c_uint64),
                 ("encode_ns", C.c_uint64), ("gpu_span_ns", C.c_uint64), ("gpu_busy_ns", C.c_uint64),
-                ("cold_wall_ns", C.c_uint64), ("infer_count", C.c_uint64), ("launches", C.c_uint64)]
+                ("cold_wall_ns", C.c_uint64), ("infer_count", C.c_uint64), ("launches", C.c_uint64),
+                ("load_done_ns", C.c_uint64), ("infer_entry_ns", C.c_uint64),
+                ("first_launch_ns", C.c_uint64), ("last_launch_ns", C.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -138,8 +140,9 @@ def kernel_name(k):
     return lib().pask_kernel_name(k).decode()
 
 
-def config(reuse=1, search=0, milestone=0, proactive=1, pdl=1, instrument=0, packaging=0):
-    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging)
+def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,
+           interleave=0):
+    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave)
 
 
 def plan(graph: Graph, cfg: Config | None = None):
@@ -166,12 +169,18 @@ class Context:
         _check(lib().pask_create(C.byref(self.h), device, C.byref(cfg) if cfg else None))
         self.n_nodes = 0
 
-    def load_model(self, graph: Graph):
+    def load_model(self, graph: Graph, plan=True):
+        """pask_load_model.  plan=False skips converting the bindings to Python
+        (keeps ctypes field access out of a timed cold window); call
+        ``bindings()`` afterwards."""
         self.n_nodes = graph.n_nodes
-        out = (Binding * max(graph.n_nodes, 1))()
-        _check(lib().pask_load_model(self.h, C.byref(graph), out))
+        self._plan_arr = (Binding * max(graph.n_nodes, 1))()
+        _check(lib().pask_load_model(self.h, C.byref(graph), self._plan_arr))
+        return self.bindings() if plan else None
+
+    def bindings(self):
         return [(b.node, b.desired_kernel, b.bound_kernel, b.how, b.lookups)
-                for b in out[:graph.n_nodes]]
+                for b in self._plan_arr[:self.n_nodes]]
 
     def infer(self, stream=0, inputs=None, outputs=None):
         ip = (C.c_void_p * len(inputs))(*inputs) if inputs else None
