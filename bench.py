@@ -188,6 +188,8 @@ def main():
                     choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
+    ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
+                    help="1: hot inferences replay a CUDA graph captured on the 2nd call")
     ap.add_argument("--packaging", type=int, default=0, choices=[0, 1],
                     help="0: one code object per kernel (default); 1: whole catalog in one")
     args = ap.parse_args()
@@ -237,7 +239,7 @@ def main():
 
     flush()
     torch.cuda.synchronize()
-    ctx = P.Context(local_rank, P.config(packaging=args.packaging))
+    ctx = P.Context(local_rank, P.config(packaging=args.packaging, graph=args.graph))
     n_nodes = len(spec["layers"])
 
     def barrier():
@@ -303,19 +305,18 @@ def main():
     hot_warm_ms = e0.elapsed_time(e1) / nw
 
     # ---------------- e2e through the public API with host buffers
-    in_host = torch.from_numpy(x.astype("float32")).pin_memory()
-    out_name = spec["outputs"][0]
-    out_dev = dm.t[out_name]
-    out_host = torch.empty(out_dev.shape, dtype=out_dev.dtype).pin_memory()
+    (in_name, _, _), = spec["inputs"]
+    in_host = torch.from_numpy(x.astype("float32")).to(dm.t[in_name].dtype).pin_memory()
+    outs_host = [torch.empty(dm.t[o].shape, dtype=dm.t[o].dtype).pin_memory() for o in spec["outputs"]]
     h2d = in_host.numel() * in_host.element_size()
-    d2h = out_host.numel() * out_host.element_size()
+    d2h = sum(o.numel() * o.element_size() for o in outs_host)
     e2e_s = []
     for i in range(args.warmup + args.steps):
         if not args.no_flush:
             flush()
         torch.cuda.synchronize()
         a = time.perf_counter()
-        ctx.infer_host([in_host.data_ptr()], [out_host.data_ptr()], sp)
+        ctx.infer_host([in_host.data_ptr()], [o.data_ptr() for o in outs_host], sp)
         b = time.perf_counter()
         if i >= args.warmup:
             e2e_s.append(b - a)
@@ -394,6 +395,8 @@ def main():
         "config": {"workload": args.workload_name, "model": args.model, "global_batch": world,
                    "per_gpu_batch": 1, "parallelism": f"replicas{world}",
                    "packaging": ["one code object per kernel", "single code object"][args.packaging],
+                   "hot_issue": "CUDA graph replay (captured on the 2nd inference)" if args.graph
+                                else "direct cuLaunchKernelEx per layer",
                    "l2": "warm (no flush)" if args.no_flush else
                          "flushed (256 MiB memset) before every timed inference"},
         "cold_ms": round(cold_max, 3),

@@ -186,6 +186,8 @@ typedef struct {
                          uploads are done while the GPU is idle anyway;
                          1 = Fig. 5 interleaving: launch each layer as soon as its kernel is
                          ready (the loader yields to the issuer)                             */
+  int32_t graph;      /* 1 = hot inferences replay a CUDA graph captured on the second call
+                         (PDL edges kept); the cold first inference always issues directly   */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;

@@ -61,6 +61,14 @@ void resolve() {
   PASK_RESOLVE(cuMemcpyHtoDAsync)
   PASK_RESOLVE(cuMemcpyDtoHAsync)
   PASK_RESOLVE(cuStreamSynchronize)
+  PASK_RESOLVE(cuStreamCreate)
+  PASK_RESOLVE(cuStreamDestroy)
+  PASK_RESOLVE(cuStreamBeginCapture)
+  PASK_RESOLVE(cuStreamEndCapture)
+  PASK_RESOLVE(cuGraphInstantiateWithFlags)
+  PASK_RESOLVE(cuGraphLaunch)
+  PASK_RESOLVE(cuGraphDestroy)
+  PASK_RESOLVE(cuGraphExecDestroy)
 #undef PASK_RESOLVE
   if (!all) {
     g_why = "a required CUDA driver entry point could not be resolved (driver too old?)";

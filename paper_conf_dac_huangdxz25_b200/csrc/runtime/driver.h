@@ -35,6 +35,14 @@ struct Driver {
   PASK_DRV_FN(cuMemcpyHtoDAsync)
   PASK_DRV_FN(cuMemcpyDtoHAsync)
   PASK_DRV_FN(cuStreamSynchronize)
+  PASK_DRV_FN(cuStreamCreate)
+  PASK_DRV_FN(cuStreamDestroy)
+  PASK_DRV_FN(cuStreamBeginCapture)
+  PASK_DRV_FN(cuStreamEndCapture)
+  PASK_DRV_FN(cuGraphInstantiateWithFlags)
+  PASK_DRV_FN(cuGraphLaunch)
+  PASK_DRV_FN(cuGraphDestroy)
+  PASK_DRV_FN(cuGraphExecDestroy)
 #undef PASK_DRV_FN
   bool ok = false;
 };

@@ -155,6 +155,9 @@ struct Ctx {
   bool pending = false;
   CUevent ev0 = nullptr, ev1 = nullptr;
   std::vector<CUevent> node_ev;
+  CUgraph graph = nullptr;          // cfg.graph: captured hot launch sequence
+  CUgraphExec graph_exec = nullptr;
+  CUstream capture_stream = nullptr;  // private non-blocking stream (legacy streams cannot capture)
   std::vector<uint64_t> node_ns;
 
   Ctx() {
@@ -721,36 +724,16 @@ PASK_API int pask_load_model(pask_ctx* c, const pask_graph* g, pask_binding* pla
   return PASK_OK;
 }
 
-PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, void* stream) {
-  t_err.clear();
-  if (!c) return set_err(PASK_EINVAL, "null ctx");
-  if (!c->have_model) return set_err(PASK_ESTATE, "pask_infer before pask_load_model");
-  int rc;
-  const bool first = c->st.infer_count == 0;
-  if (first) c->st.infer_entry_ns = now_ns() - c->t_entry;
-  for (size_t i = 0; inputs && i < c->inputs.size(); ++i)
-    if (inputs[i] && (rc = rebind(c, c->inputs[i], inputs[i]))) return rc;
-  for (size_t i = 0; outputs && i < c->outputs.size(); ++i)
-    if (outputs[i] && (rc = rebind(c, c->outputs[i], outputs[i]))) return rc;
+namespace pask {
+namespace {
+// Issue every node's launch on stream s (the issue loop, PAPER.md:95 I_i).
+int issue_all(Ctx* c, CUstream s, bool first) {
   const Driver* d = c->d;
-  CUstream s = static_cast<CUstream>(stream);
+  int rc;
   CUlaunchAttribute attr[2];
-  if (c->cfg.proactive && !c->cfg.interleave) {
-    // load-first: every planned kernel uploaded before the first launch (uploads
-    // wait for running GPU work, so interleaving them with launches only
-    // serialises each upload behind the layers already queued)
-    for (int32_t k : c->plan.loaded)
-      if ((rc = wait_kernel(c, k))) return rc;
-  }
-  c->issuing.store(1, std::memory_order_release);
-  struct Idle {  // the loader may run again once this inference is issued (or fails)
-    std::atomic<int32_t>& f;
-    ~Idle() { f.store(0, std::memory_order_release); }
-  } idle{c->issuing};
   for (size_t i = 0; i < c->launches.size(); ++i) {
     Launch& L = c->launches[i];
     if ((rc = wait_kernel(c, L.kernel))) return rc;
-    if (i == 0) d->cuEventRecord(c->ev0, s);
     if (c->cfg.instrument) d->cuEventRecord(c->node_ev[2 * i], s);
     CUlaunchConfig cfg{};
     cfg.gridDimX = L.grid[0];
@@ -786,6 +769,98 @@ PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, 
     if (c->cfg.instrument) d->cuEventRecord(c->node_ev[2 * i + 1], s);
     c->st.launches++;
     if (first && i == 0) c->st.first_launch_ns = now_ns() - c->t_entry;
+  }
+  return PASK_OK;
+}
+
+void drop_graph(Ctx* c) {
+  if (c->graph_exec) c->d->cuGraphExecDestroy(c->graph_exec);
+  if (c->graph) c->d->cuGraphDestroy(c->graph);
+  c->graph_exec = nullptr;
+  c->graph = nullptr;
+}
+
+// Capture the launch sequence into a CUDA graph (hot path) on the private
+// capture stream; the executable graph is then launched on the caller's stream.
+int capture_graph(Ctx* c) {
+  const Driver* d = c->d;
+  drop_graph(c);
+  CUresult r;
+  if (!c->capture_stream) {
+    r = d->cuStreamCreate(&c->capture_stream, CU_STREAM_NON_BLOCKING);
+    if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuStreamCreate"));
+  }
+  CUstream s = c->capture_stream;
+  r = d->cuStreamBeginCapture(s, CU_STREAM_CAPTURE_MODE_THREAD_LOCAL);
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuStreamBeginCapture"));
+  const uint64_t launches = c->st.launches;
+  int rc = issue_all(c, s, false);
+  c->st.launches = launches;  // captured, not launched
+  CUgraph g = nullptr;
+  r = d->cuStreamEndCapture(s, &g);
+  if (rc) {
+    if (g) d->cuGraphDestroy(g);
+    return rc;
+  }
+  if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuStreamEndCapture"));
+  CUgraphExec ge = nullptr;
+  r = d->cuGraphInstantiateWithFlags(&ge, g, 0);
+  if (r != CUDA_SUCCESS) {
+    d->cuGraphDestroy(g);
+    return set_err(PASK_ECUDA, cu_err(d, r, "cuGraphInstantiateWithFlags"));
+  }
+  c->graph = g;
+  c->graph_exec = ge;
+  return PASK_OK;
+}
+}  // namespace
+}  // namespace pask
+
+PASK_API int pask_infer(pask_ctx* c, void* const* inputs, void* const* outputs, void* stream) {
+  t_err.clear();
+  if (!c) return set_err(PASK_EINVAL, "null ctx");
+  if (!c->have_model) return set_err(PASK_ESTATE, "pask_infer before pask_load_model");
+  int rc;
+  const bool first = c->st.infer_count == 0;
+  if (first) c->st.infer_entry_ns = now_ns() - c->t_entry;
+  bool rebound = false;
+  for (size_t i = 0; inputs && i < c->inputs.size(); ++i)
+    if (inputs[i] && c->tensors[c->inputs[i]].dptr != inputs[i]) {
+      if ((rc = rebind(c, c->inputs[i], inputs[i]))) return rc;
+      rebound = true;
+    }
+  for (size_t i = 0; outputs && i < c->outputs.size(); ++i)
+    if (outputs[i] && c->tensors[c->outputs[i]].dptr != outputs[i]) {
+      if ((rc = rebind(c, c->outputs[i], outputs[i]))) return rc;
+      rebound = true;
+    }
+  const Driver* d = c->d;
+  CUstream s = static_cast<CUstream>(stream);
+  if (c->cfg.proactive && !c->cfg.interleave) {
+    // load-first: every planned kernel uploaded before the first launch (uploads
+    // wait for running GPU work, so interleaving them with launches only
+    // serialises each upload behind the layers already queued)
+    for (int32_t k : c->plan.loaded)
+      if ((rc = wait_kernel(c, k))) return rc;
+  }
+  c->issuing.store(1, std::memory_order_release);
+  struct Idle {  // the loader may run again once this inference is issued (or fails)
+    std::atomic<int32_t>& f;
+    ~Idle() { f.store(0, std::memory_order_release); }
+  } idle{c->issuing};
+  const bool use_graph = c->cfg.graph && !c->cfg.instrument && !first;
+  if (use_graph && (rebound || !c->graph_exec)) {
+    if ((rc = capture_graph(c))) return rc;
+  }
+  d->cuEventRecord(c->ev0, s);
+  if (use_graph) {
+    const uint64_t t0 = now_ns();
+    CUresult r = d->cuGraphLaunch(c->graph_exec, s);
+    c->st.issue_ns += now_ns() - t0;
+    if (r != CUDA_SUCCESS) return set_err(PASK_ECUDA, cu_err(d, r, "cuGraphLaunch"));
+    c->st.launches += c->launches.size();
+  } else if ((rc = issue_all(c, s, first))) {
+    return rc;
   }
   if (first) {
     c->st.last_launch_ns = now_ns() - c->t_entry;
@@ -910,6 +985,8 @@ PASK_API int pask_destroy(pask_ctx* c) {
     if (e) d->cuEventDestroy(e);
   if (c->ev0) d->cuEventDestroy(c->ev0);
   if (c->ev1) d->cuEventDestroy(c->ev1);
+  drop_graph(c);
+  if (c->capture_stream) d->cuStreamDestroy(c->capture_stream);
   if (c->lib) d->cuLibraryUnload(c->lib);
   for (CUlibrary l : c->klib)
     if (l) d->cuLibraryUnload(l);

@@ -52,6 +52,7 @@ pask_config default_config() {
   c.instrument = 0;
   c.packaging = 0;
   c.interleave = 0;
+  c.graph = 0;
   return c;
 }
 

@@ -56,7 +56,7 @@ class Graph(C.Structure):
 class Config(C.Structure):
     _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
                 ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
-                ("packaging", C.c_int32), ("interleave", C.c_int32)]
+                ("packaging", C.c_int32), ("interleave", C.c_int32), ("graph", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -141,8 +141,8 @@ def kernel_name(k):
 
 
 def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,
-           interleave=0):
-    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave)
+           interleave=0, graph=0):
+    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph)
 
 
 def plan(graph: Graph, cfg: Config | None = None):
