@@ -199,20 +199,13 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const uint32_t tmem_base = *tmem_slot;
   if (trace && t == 0) trace[1] = globaltimer();
 
-  pdl_wait();               // inputs of this layer are complete and visible
   pdl_launch_dependents();  // let the next layer's prologue start
-  if (trace && t == 0) trace[2] = globaltimer();
+  // griddepcontrol.wait is per role: weights (B, bias) do not depend on the
+  // previous layer, so they are fetched before it; activations after it.
 
   if (warp == 4) {
     // ================= TMA producer
     if (lane == 0) {
-      if (res_tma) {  // residual rows [r0, r0 + rows_per) of the tile, consumed by the epilogue
-        mbar_arrive_expect_tx(res_bar, static_cast<uint32_t>(rows_per * bn * 2));
-#pragma unroll 1
-        for (int j = 0; j < bn / box_cols; ++j)
-          tma_load_3d(ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), &p.tmap_r, res_bar,
-                      n0 + j * box_cols, m0 + r0, b);
-      }
       // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
       int iw = 0, ih = 0, in = 0, cc = 0, tr = 0, ts = 0;
       const int cpt = p.C >> 6;  // 64-channel chunks per filter tap
@@ -229,14 +222,40 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         tr = tap / p.S;
         ts = tap - tr * p.S;
       }
+      // weights of the first min(nk, stages) k-blocks before griddepcontrol.wait
+      // (they overlap the previous layer's tail); ring slots start empty.  An
+      // activation B operand (attention QK^T / PV) must wait like A.
+      const int pre = p.b_const ? min(nk, stages) : 0;
+      for (int i = 0; i < pre; ++i) {
+        const uint32_t sb = smem_base + i * stage_bytes + kABytes;
+        const int kb = kb_begin + i;
+        mbar_arrive_expect_tx(full0 + 8 * i, b_bytes + (gather ? 0u : kABytes));
+        if (p.b_major == 0) {
+          tma_load_3d(sb, &p.tmap_b, full0 + 8 * i, kb * kBK, n0, b);
+        } else {
+#pragma unroll 1
+          for (int j = 0; j < bn / 64; ++j)
+            tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * i, n0 + j * 64, kb * kBK, b);
+        }
+      }
+      pdl_wait();  // activations / residual of this layer are complete and visible
+      if (trace) trace[2] = globaltimer();
+      if (res_tma) {  // residual rows [r0, r0 + rows_per) of the tile, consumed by the epilogue
+        mbar_arrive_expect_tx(res_bar, static_cast<uint32_t>(rows_per * bn * 2));
+#pragma unroll 1
+        for (int j = 0; j < bn / box_cols; ++j)
+          tma_load_3d(ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), &p.tmap_r, res_bar,
+                      n0 + j * box_cols, m0 + r0, b);
+      }
       int s = 0;
       uint32_t ph = 0;
       for (int i = 0; i < nk; ++i) {
-        mbar_wait(empty0 + 8 * s, ph ^ 1);
+        const bool b_done = i < pre;
+        if (!b_done) mbar_wait(empty0 + 8 * s, ph ^ 1);
         const uint32_t sa = smem_base + s * stage_bytes;
         const uint32_t sb = sa + kABytes;
         const int kb = kb_begin + i;
-        mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
+        if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
         if (kAllowGather && im2col) {
           tma_load_im2col_4d(sa, &p.tmap_a, full0 + 8 * s, cc * 64, iw, ih, in,
                              static_cast<uint16_t>(ts * p.dw), static_cast<uint16_t>(tr * p.dh));
@@ -250,12 +269,14 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         } else if (!gather) {
           tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
         }
-        if (p.b_major == 0) {
-          tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
-        } else {
+        if (!b_done) {
+          if (p.b_major == 0) {
+            tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
+          } else {
 #pragma unroll 1
-          for (int j = 0; j < bn / 64; ++j)
-            tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * s, n0 + j * 64, kb * kBK, b);
+            for (int j = 0; j < bn / 64; ++j)
+              tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * s, n0 + j * 64, kb * kBK, b);
+          }
         }
         if (++s == stages) {
           s = 0;
@@ -298,6 +319,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   } else {
     // ================= warps 0-3: bias, (gather), epilogue
     if (t < bn) s_bias[t] = (p.bias != nullptr && n0 + t < p.N) ? __ldg(p.bias + n0 + t) : 0.f;
+    pdl_wait();  // before reading this layer's activations (gather) or writing outputs
     if (kAllowGather && gather) {
       // implicit im2col: lane t owns 16 B chunk j = t % 8 of rows rg + 16 * ri
       const int j = t & 7;
@@ -421,14 +443,30 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
     if (res_tma) mbar_wait(res_bar, 0);
     // items: (row, 16-column chunk).  splits == 1: thread t owns TMEM lane / row t.
     // splits > 1: the 128 threads stride over this rank's rows_per x cpr items.
+    // items: (row, 16-column chunk).  splits == 1: thread t owns TMEM lane / row t
+    // and reads 32 columns per tcgen05.ld; splits > 1: the 128 threads stride
+    // over this rank's rows_per x cpr items and reduce the S receive slots.
     const int n_items = splits == 1 ? cpr : (rows_per * cpr - t + 127) / 128;
+    float buf[32];
     for (int k = 0; k < n_items; ++k) {
       int row, cb;
       float v[16];
       if (splits == 1) {
         row = t;
         cb = k << 4;
-        tmem_ld16(taddr + cb, v);  // warp-collective
+        const bool odd = (k & 1) != 0;
+        if (!odd) {
+          if (cb + 32 <= bn) {
+            tmem_ld32(taddr + cb, buf);  // warp-collective
+          } else {
+            float h[16];
+            tmem_ld16(taddr + cb, h);
+#pragma unroll
+            for (int i = 0; i < 16; ++i) buf[i] = h[i];
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = odd ? buf[16 + i] : buf[i];
       } else {
         const int it = t + 128 * k;
         const int lr = it / cpr;  // row within this rank's slice

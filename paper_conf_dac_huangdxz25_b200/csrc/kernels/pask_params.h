@@ -41,6 +41,7 @@ struct alignas(64) GemmParams {
   int32_t stages;        // smem pipeline depth
   int32_t a_mode;        // AMode
   int32_t b_major;       // 0 K-major, 1 MN-major
+  int32_t b_const;       // 1: B is weights (fetched before griddepcontrol.wait); 0: B is an activation
   int32_t act;           // pask_act
   int32_t m_tiles, n_tiles;
   int32_t c_tma;         // 1: output (and residual) through TMA + smem staging

@@ -375,6 +375,7 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
       q.num_kb = t.num_kb; q.kb_per_split = (t.num_kb + t.splits - 1) / t.splits; q.splits = t.splits;
       q.rows_per = t.rows_per; q.c_tma = c_tma;
       q.bn = t.bn; q.stages = t.stages; q.b_major = b_major; q.act = nd.act;
+      q.b_const = (p.op == OC_CONV || nd.w != nullptr) ? 1 : 0;
       q.m_tiles = t.m_tiles; q.n_tiles = t.n_tiles;
       q.idesc = make_idesc(t.bn, b_major);
       q.tmem_cols = t.tmem_cols;
@@ -455,10 +456,13 @@ int lower_node(Ctx* c, int32_t i, std::string* err) {
                          static_cast<uint64_t>(nd.stride_b) * 2, 64, 64, err);
         if (rc) return rc;
       }
-      {  // debug-only phase trace (PASK_TRACE_NODE=i PASK_TRACE_PTR=<device address>)
+      {  // debug-only phase trace (PASK_TRACE_NODE=i or -1 for all; PASK_TRACE_PTR=<device
+         // address>; node i writes 8 stamps per CTA at PTR + i * 8 * 4096 words)
         const char* tn = getenv("PASK_TRACE_NODE");
         const char* tp = getenv("PASK_TRACE_PTR");
-        if (tn && tp && atoi(tn) == i) q.trace = reinterpret_cast<unsigned long long*>(strtoull(tp, nullptr, 0));
+        if (tn && tp && (atoi(tn) == i || atoi(tn) == -1))
+          q.trace = reinterpret_cast<unsigned long long*>(strtoull(tp, nullptr, 0)) +
+                    (atoi(tn) == -1 ? static_cast<size_t>(i) * 8 * 4096 : 0);
       }
       L.block[0] = kGemmThreads;
       L.grid[0] = static_cast<unsigned>(t.m_tiles);

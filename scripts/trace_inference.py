@@ -1,0 +1,57 @@
+"""Debug: GPU timeline of one hot inference (PDL on, direct issue): per
+contraction node, first CTA start / last CTA end and median phase times."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_dac_huangdxz25_b200 import pask as P  # noqa: E402
+from paper_conf_dac_huangdxz25_b200.model import DeviceModel  # noqa: E402
+from workloads import build_model  # noqa: E402
+
+name = sys.argv[1] if len(sys.argv) > 1 else "resnet50"
+spec, x = build_model(name)
+dm = DeviceModel(spec)
+dm.set_input(x)
+n = len(spec["layers"])
+buf = torch.zeros(n * 8 * 4096, dtype=torch.int64, device="cuda")
+os.environ["PASK_TRACE_NODE"] = "-1"
+os.environ["PASK_TRACE_PTR"] = str(buf.data_ptr())
+ctx = P.Context(0, P.config())
+ctx.load_model(dm.graph)
+s = torch.cuda.current_stream().cuda_stream
+for _ in range(5):
+    ctx.infer(s)
+ctx.sync()
+buf.zero_()
+torch.cuda.synchronize()
+ctx.infer(s)
+ctx.sync()
+torch.cuda.synchronize()
+tr = buf.view(n, 4096, 8).cpu().numpy().astype(np.float64)
+plan = ctx.bindings()
+t0 = None
+rows = []
+for i in range(n):
+    t = tr[i]
+    t = t[t[:, 0] > 0]
+    if not len(t):
+        continue
+    if t0 is None:
+        t0 = t[:, 0].min()
+    rel = (t - t0) / 1e3
+    rows.append((i, len(t), rel[:, 0].min(), rel[:, 7].max(), np.median(rel[:, 2] - rel[:, 0]),
+                 np.median(rel[:, 3] - rel[:, 2]), np.median(rel[:, 5] - rel[:, 3]),
+                 np.median(rel[:, 6] - rel[:, 5]), np.median(rel[:, 7] - rel[:, 6])))
+prev_end = None
+print(f"{'node':>4} {'ctas':>4} {'start':>8} {'end':>8} {'dur':>6} {'gap':>6} | pre-wait first-load mainloop epilogue store (median us)")
+for r in rows:
+    i, nc, st, en = r[:4]
+    gap = st - prev_end if prev_end is not None else 0.0
+    L = spec["layers"][i]
+    desc = L["op"] + (str(tuple(L["w"].shape)) + f" s{L['stride'][0]}" if L["op"] == "conv" else "")
+    print(f"{i:4d} {nc:4d} {st:8.2f} {en:8.2f} {en-st:6.2f} {gap:6.2f} | {r[4]:5.2f} {r[5]:5.2f} {r[6]:5.2f} {r[7]:5.2f} {r[8]:5.2f}  {desc}")
+    prev_end = en
+print("total span of traced nodes (us):", rows[-1][3] - rows[0][2])
