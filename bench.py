@@ -161,7 +161,7 @@ def run_reference(args, spec, x, rank):
     w = time_oracle(spec, x, max(args.warmup, 0), 60.0) if args.warmup else []
     ts = time_oracle(spec, x, args.steps, 240.0)
     mean_s = statistics.mean(ts)
-    val = 1.0 / mean_s
+    val = args.batch / mean_s
     line = {
         "impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "imgs/s",
         "n_gpus": args.gpus, "steps": len(ts), "warmup": len(w), "ms_per_step": round(1e3 * mean_s, 2),
@@ -170,7 +170,7 @@ def run_reference(args, spec, x, rank):
                                         "model": args.model},
         "cpu_baseline": {"value": round(val, 4), "unit": "imgs/s", "cores": cores_used(),
                          "kind": "oracle",
-                         "sample": f"{len(ts)} full fp64 numpy-oracle forwards of one image"},
+                         "sample": f"{len(ts)} full fp64 numpy-oracle forwards of a batch-{args.batch} input"},
         "e2e": {"value": round(val, 4), "unit": "imgs/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -186,6 +186,7 @@ def main():
     ap.add_argument("--impl", default="pask", choices=["pask", "reference"])
     ap.add_argument("--model", default="resnet50",
                     choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"])
+    ap.add_argument("--batch", type=int, default=1, help="images per inference (Table II sweep)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
@@ -211,7 +212,7 @@ def main():
         dist.init_process_group("gloo", rank=rank, world_size=world)
 
     from workloads import build_model
-    spec, x = build_model(args.model)
+    spec, x = build_model(args.model, **({"batch": args.batch} if args.batch != 1 else {}))
 
     if args.impl == "reference":
         run_reference(args, spec, x, rank)
@@ -374,14 +375,14 @@ def main():
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         ts = time_oracle(spec, x, 5, 20.0)
-        cpu = {"value": round(1.0 / statistics.mean(ts), 4), "unit": "imgs/s", "cores": cores_used(),
+        cpu = {"value": round(args.batch / statistics.mean(ts), 4), "unit": "imgs/s", "cores": cores_used(),
                "kind": "oracle",
-               "sample": f"{len(ts)} full fp64 numpy-oracle forwards of one {args.model} image"}
+               "sample": f"{len(ts)} full fp64 numpy-oracle forwards of a batch-{args.batch} {args.model} input"}
 
     st = cold_stats
     line = {
         "metric": METRIC,
-        "value": round(world * 1000.0 / hot_max, 2),
+        "value": round(world * args.batch * 1000.0 / hot_max, 2),
         "unit": "imgs/s",
         "n_gpus": world,
         "steps": args.steps,
@@ -392,8 +393,9 @@ def main():
         "vs_baseline": None,
         "dtype": "bf16",
         "data": "synthetic (seeded N(0,1) input, random-init weights of the architecture)",
-        "config": {"workload": args.workload_name, "model": args.model, "global_batch": world,
-                   "per_gpu_batch": 1, "parallelism": f"replicas{world}",
+        "config": {"workload": args.workload_name, "model": args.model,
+                   "global_batch": world * args.batch, "per_gpu_batch": args.batch,
+                   "parallelism": f"replicas{world}",
                    "packaging": ["one code object per kernel", "single code object"][args.packaging],
                    "hot_issue": "CUDA graph replay (captured on the 2nd inference)" if args.graph
                                 else "direct cuLaunchKernelEx per layer",
@@ -418,7 +420,7 @@ def main():
                               "cold_wall": round(st["cold_wall_ns"] / 1e3, 1)},
         "load_timeline_us": timeline,
         "per_kernel_ms": {k: round(v["ms"], 4) for k, v in per_kernel.items()},
-        "e2e": {"value": round(world * 1000.0 / e2e_max, 2), "unit": "imgs/s",
+        "e2e": {"value": round(world * args.batch * 1000.0 / e2e_max, 2), "unit": "imgs/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": round(e2e_max, 4)},
         "gpu_launches": n_nodes * args.steps,

@@ -32,13 +32,13 @@ SCHEMES = {
 }
 
 
-def child(model, scheme):
+def child(model, scheme, batch=1):
     import torch
 
     from paper_conf_dac_huangdxz25_b200 import pask as P
     from paper_conf_dac_huangdxz25_b200.model import DeviceModel
     from workloads import build_model
-    spec, x = build_model(model)
+    spec, x = build_model(model, **({"batch": batch} if batch != 1 else {}))
     dm = DeviceModel(spec)
     dm.set_input(x)
     torch.cuda.synchronize()
@@ -85,15 +85,17 @@ def main():
     ap.add_argument("--n", type=int, default=20)
     ap.add_argument("--schemes", default=",".join(SCHEMES))
     ap.add_argument("--child", default=None)
+    ap.add_argument("--batch", type=int, default=1)
     a = ap.parse_args()
     if a.child:
-        child(a.model, a.child)
+        child(a.model, a.child, a.batch)
         return
     out = {}
     for scheme in a.schemes.split(","):
         samples = []
         for _ in range(a.n):
-            r = subprocess.run([sys.executable, __file__, "--model", a.model, "--child", scheme],
+            r = subprocess.run([sys.executable, __file__, "--model", a.model, "--child", scheme,
+                                "--batch", str(a.batch)],
                                capture_output=True, text=True, timeout=300)
             line = [l for l in r.stdout.splitlines() if l.startswith("{")]
             if not line:

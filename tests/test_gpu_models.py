@@ -34,6 +34,34 @@ def test_model_layers_teacher_forced(name):
     ctx.close()
 
 
+@pytest.mark.parametrize("name,batch", [("resnet50", 3), ("mobilenet_v2", 2), ("tiny_cnn", 5)])
+def test_batched_models_teacher_forced(name, batch):
+    """Batch > 1 (Table II sweep): pixels of several
+    images share GEMM tiles (gather / TMA im2col wrap across images)."""
+    spec, x = build_model(name, batch=batch)
+    dm, ctx, plan = run_model(spec, x)
+    errs = teacher_forced_errors(dm, spec, x)
+    bad = [(i, op, e) for i, op, e in errs if not e <= TOL]
+    assert not bad, f"layers over tolerance: {bad[:10]}"
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", ["resnet50", "bert_base"])
+def test_graph_replay_bitwise(name):
+    """Hot inferences replayed from a captured CUDA graph equal direct issue, bitwise."""
+    import torch
+    spec, x = build_model(name)
+    dm, ctx, _ = run_model(spec, x, cfg=P.config(graph=1))
+    ref = [dm.read_raw(n) for n in spec["outputs"]]
+    s = torch.cuda.current_stream().cuda_stream
+    for _ in range(3):
+        ctx.infer(s)
+    ctx.sync()
+    for a, n in zip(ref, spec["outputs"]):
+        np.testing.assert_array_equal(a, dm.read_raw(n))
+    ctx.close()
+
+
 @pytest.mark.parametrize("packaging", [0, 1])
 @pytest.mark.parametrize("cfg", ["reactive", "pask_i", "pask_r", "no_pdl"])
 def test_schemes_same_outputs(cfg, packaging):

@@ -182,9 +182,9 @@ class _Builder:
 # ---------------------------------------------------------------------------
 # C1 tiny CNN (BASELINE.json configs[0])
 # ---------------------------------------------------------------------------
-def tiny_cnn(seed_weights=1, hw=32):
+def tiny_cnn(seed_weights=1, hw=32, batch=1):
     b = _Builder("tiny_cnn", seed_weights)
-    x = b.input((1, 3, hw, hw), "f32")
+    x = b.input((batch, 3, hw, hw), "f32")
     t = b.layout(x)
     t = b.conv(t, 16, 3, 1, 1, act="relu")
     t = b.conv(t, 32, 3, 1, 1, act="relu")
