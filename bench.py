@@ -260,12 +260,12 @@ def main():
     cold_ms = cold_stats["cold_wall_ns"] / 1e6      # library clock: load_model entry -> sync return
     cold_py_ms = (t1 - t0) / 1e6                    # the same window seen from Python
     timeline = {}
-    for k in range(P.NUM_KERNELS):
+    for k in range(P.num_kernels()):
         ld, rd, lb = ctx.kernel_timeline(k)
         if ld:
             timeline[P.kernel_name(k)] = {"load_us": round(ld / 1e3, 1), "ready_at_us": round(rd / 1e3, 1),
                                           "lib_us": round(lb / 1e3, 1)}
-    loaded = sorted(P.kernel_name(k) for k in range(P.NUM_KERNELS) if ctx.kernel_is_loaded(k))
+    loaded = sorted(P.kernel_name(k) for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k))
 
     # ---------------- warmup
     for _ in range(args.warmup):

@@ -98,8 +98,14 @@ typedef enum {
   PASK_K_GEMM = 6,       /* batched GEMM, tcgen05/TMEM; cat (GEMM, bf16, ROWMAJOR)      */
   PASK_K_SOFTMAX = 7,    /* cat (SOFTMAX, bf16, ROWMAJOR)                               */
   PASK_K_LAYERNORM = 8,  /* cat (LAYERNORM, bf16, ROWMAJOR)                             */
-  PASK_NUM_KERNELS = 9
+  PASK_NUM_KERNELS = 9   /* size of the generic catalog; ids >= 9 are the per-problem
+                            specialised conv solutions of the tuned catalog (one per
+                            (R, S, stride, pad, dilation, C) of configs C1-C3, category
+                            (CONV, bf16, NHWC), applicable to exactly that problem
+                            shape); pask_num_kernels() returns the total            */
 } pask_kernel_id;
+
+#define PASK_MAX_KERNELS 64
 
 /* A tensor: logical dims (n, h, w, c), element type, memory order, and a
  * caller-owned device pointer (16-byte aligned). */
@@ -188,6 +194,9 @@ typedef struct {
                          ready (the loader yields to the issuer)                             */
   int32_t graph;      /* 1 = hot inferences replay a CUDA graph captured on the second call
                          (PDL edges kept); the cold first inference always issues directly   */
+  int32_t catalog;    /* 0 = generic catalog; 1 = tuned catalog: s* of a dense conv is its
+                         per-problem specialised solution when one exists (the library
+                         behaviour PASK starts from; the Baseline scheme)       */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;
@@ -303,7 +312,7 @@ int pask_destroy(pask_ctx *ctx);
 /* Thread-local description of the last error on this thread ("" if none). */
 const char *pask_last_error(void);
 
-/* Catalog introspection (host only). */
+/* Catalog introspection (host only): total kernels (generic + specialised). */
 int32_t pask_num_kernels(void);
 const char *pask_kernel_name(int32_t kernel_id);
 

@@ -31,6 +31,18 @@ K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN = ra
 KERNEL_NAMES = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw",
                 "pask_pool", "pask_pool_gavg", "pask_gemm", "pask_softmax", "pask_layernorm"]
 
+# Tuned catalog: one specialised conv solution per distinct dense
+# conv problem (R, S, stride, pad, dilation, C) of configs C1-C3, ids 9 + i in
+# sorted order; applicable to exactly that shape (any K, N, H, W).
+SPECS = sorted([
+    (1, 1, 1, 0, 1, c) for c in (16, 24, 32, 64, 96, 128, 144, 160, 192, 256, 320, 384, 512, 576,
+                                 960, 1024, 2048)
+] + [(1, 1, 2, 0, 1, c) for c in (256, 512, 1024)]
+  + [(3, 3, 1, 1, 1, c) for c in (8, 16, 32, 64, 128, 256, 512)]
+  + [(3, 3, 2, 1, 1, c) for c in (8, 128, 256, 512)] + [(7, 7, 2, 3, 1, 8)])
+N_GENERIC = 9
+KERNEL_NAMES = KERNEL_NAMES + ["pask_conv_spec_r%ds%du%dp%dd%dc%d" % sp for sp in SPECS]
+
 # category key (op class, dtype, layout): dtype 0 = bf16 compute path, layouts
 # 0 NCHW, 1 NHWC, 2 row-major
 CATEGORY = {
@@ -44,6 +56,7 @@ CATEGORY = {
     K_SOFTMAX: (SOFTMAX, 0, 2),
     K_LN: (LAYERNORM, 0, 2),
 }
+CATEGORY.update({N_GENERIC + i: (CONV, 0, 1) for i in range(len(SPECS))})
 
 
 def _conv_class(p):
@@ -53,6 +66,12 @@ def _conv_class(p):
 def is_applicable(kid, p):
     """IsApplicable(kernel, problem) -- PAPER.md:83, Alg. 1 l.15."""
     op = p["op"]
+    if kid >= N_GENERIC:
+        r, s, st, pd, dl, c = SPECS[kid - N_GENERIC]
+        return (op == CONV and p["r"] == r and p["s"] == s and p["stride_h"] == st
+                and p["stride_w"] == st and p["pad_h"] == pd and p["pad_w"] == pd
+                and p["dil_h"] == dl and p["dil_w"] == dl and p["c"] == c and p["k"] % 8 == 0
+                and p["p"] >= 1 and p["q"] >= 1)
     if kid == K_LAYOUT:
         return (op == LAYOUT and p["k"] % 8 == 0 and p["c"] <= p["k"]
                 and p["n"] * p["h"] * p["w"] * max(p["c"], p["k"]) < 2 ** 31)
@@ -92,9 +111,14 @@ def is_applicable(kid, p):
     raise ValueError(kid)
 
 
-def static_choice(p):
-    """s*_i: the library's statically 'best' (most specialised) solution."""
+def static_choice(p, catalog="generic"):
+    """s*_i: the library's statically 'best' (most specialised) solution.
+    With the tuned catalog a dense conv's s* is its own specialised solution."""
     op = p["op"]
+    if catalog == "tuned" and op == CONV:
+        for i in range(len(SPECS)):
+            if is_applicable(N_GENERIC + i, p):
+                return N_GENERIC + i
     if op == LAYOUT:
         return K_LAYOUT
     if op == DWCONV:
@@ -189,7 +213,7 @@ def problems_from_spec(spec):
 DIRECT, REUSED, LOADED = 0, 1, 2
 
 
-def execution_plan(problems, reuse=True, search="categorical", milestone=0):
+def execution_plan(problems, reuse=True, search="categorical", milestone=0, catalog="generic"):
     """Algorithm 1 EXECUTIONPLAN for layers 1..n.
 
     Returns dict(bindings=[(node, desired, bound, how, lookups)], loaded=[ids in load
@@ -210,7 +234,7 @@ def execution_plan(problems, reuse=True, search="categorical", milestone=0):
         touch(kid)
 
     for i, p in enumerate(problems):
-        s_star = static_choice(p)
+        s_star = static_choice(p, catalog)
         if not is_applicable(s_star, p):
             raise ValueError(f"node {i}: s* {KERNEL_NAMES[s_star]} not applicable")
         layer_no = i + 1

@@ -123,7 +123,40 @@ __device__ __forceinline__ void epi16(const GemmParams& p, const EpiCtx& e, int 
   }
 }
 
-template <bool kAllowGather>
+// Geometry policy of the contraction body.  DynGeo reads filter size, stride,
+// padding, dilation, input channels and the A-operand path from the parameter
+// block (the generic, reusable kernels); FixGeo bakes them in at compile time
+// (the per-problem specialised solutions of the paper's Baseline, PAPER.md:83
+// Fig. 4: smaller, branch-free code that is applicable to one problem shape).
+struct DynGeo {
+  __device__ static int R(const GemmParams& p) { return p.R; }
+  __device__ static int S(const GemmParams& p) { return p.S; }
+  __device__ static int SH(const GemmParams& p) { return p.sh; }
+  __device__ static int SW(const GemmParams& p) { return p.sw; }
+  __device__ static int PH(const GemmParams& p) { return p.ph; }
+  __device__ static int PW(const GemmParams& p) { return p.pw; }
+  __device__ static int DH(const GemmParams& p) { return p.dh; }
+  __device__ static int DW(const GemmParams& p) { return p.dw; }
+  __device__ static int C(const GemmParams& p) { return p.C; }
+  __device__ static int amode(const GemmParams& p) { return p.a_mode; }
+};
+template <int R_, int S_, int ST_, int PD_, int DL_, int C_>
+struct FixGeo {
+  __device__ static constexpr int R(const GemmParams&) { return R_; }
+  __device__ static constexpr int S(const GemmParams&) { return S_; }
+  __device__ static constexpr int SH(const GemmParams&) { return ST_; }
+  __device__ static constexpr int SW(const GemmParams&) { return ST_; }
+  __device__ static constexpr int PH(const GemmParams&) { return PD_; }
+  __device__ static constexpr int PW(const GemmParams&) { return PD_; }
+  __device__ static constexpr int DH(const GemmParams&) { return DL_; }
+  __device__ static constexpr int DW(const GemmParams&) { return DL_; }
+  __device__ static constexpr int C(const GemmParams&) { return C_; }
+  __device__ static constexpr int amode(const GemmParams&) {
+    return (R_ == 1 && S_ == 1 && ST_ == 1 && PD_ == 0) ? A_TMA : (C_ % 64 == 0 ? A_IM2COL : A_GATHER);
+  }
+};
+
+template <bool kAllowGather, class Geo = DynGeo>
 __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -155,8 +188,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const uint32_t ro = smem_base + reg0;
   const uint32_t recv = smem_base + ring_bytes;  // slot s: rows [s*rows_per, (s+1)*rows_per)
 
-  const bool gather = kAllowGather && (p.a_mode == A_GATHER);
-  const bool im2col = kAllowGather && (p.a_mode == A_IM2COL);
+  const int a_mode = Geo::amode(p);
+  const bool gather = kAllowGather && (a_mode == A_GATHER);
+  const bool im2col = kAllowGather && (a_mode == A_IM2COL);
+  const int gR = Geo::R(p), gS = Geo::S(p), gSH = Geo::SH(p), gSW = Geo::SW(p);
+  const int gPH = Geo::PH(p), gPW = Geo::PW(p), gDH = Geo::DH(p), gDW = Geo::DW(p), gC = Geo::C(p);
+  (void)gR;
   const int mt = blockIdx.x, nt = blockIdx.y;
   const int b = blockIdx.z / splits;
   const int split = blockIdx.z - b * splits;
@@ -208,19 +245,19 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
     if (lane == 0) {
       // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
       int iw = 0, ih = 0, in = 0, cc = 0, tr = 0, ts = 0;
-      const int cpt = p.C >> 6;  // 64-channel chunks per filter tap
+      const int cpt = gC >> 6;  // 64-channel chunks per filter tap
       if (kAllowGather && im2col) {
         const int pq = p.P * p.Q;
         in = m0 / pq;
         const int rem = m0 - in * pq;
         const int pp = rem / p.Q;
         const int qq = rem - pp * p.Q;
-        iw = qq * p.sw - p.pw;
-        ih = pp * p.sh - p.ph;
+        iw = qq * gSW - gPW;
+        ih = pp * gSH - gPH;
         const int tap = kb_begin / cpt;
         cc = kb_begin - tap * cpt;
-        tr = tap / p.S;
-        ts = tap - tr * p.S;
+        tr = tap / gS;
+        ts = tap - tr * gS;
       }
       // weights of the first min(nk, stages) k-blocks before griddepcontrol.wait
       // (they overlap the previous layer's tail); ring slots start empty.  An
@@ -258,10 +295,10 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
         if (kAllowGather && im2col) {
           tma_load_im2col_4d(sa, &p.tmap_a, full0 + 8 * s, cc * 64, iw, ih, in,
-                             static_cast<uint16_t>(ts * p.dw), static_cast<uint16_t>(tr * p.dh));
+                             static_cast<uint16_t>(ts * gDW), static_cast<uint16_t>(tr * gDH));
           if (++cc == cpt) {
             cc = 0;
-            if (++ts == p.S) {
+            if (++ts == gS) {
               ts = 0;
               ++tr;
             }
@@ -338,8 +375,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
 #pragma unroll
         for (int ri = 0; ri < 8; ++ri) {
           rv[ri] = (m + 16 * ri) < p.M;
-          ih0[ri] = pp * p.sh - p.ph;
-          iw0[ri] = qq * p.sw - p.pw;
+          ih0[ri] = pp * gSH - gPH;
+          iw0[ri] = qq * gSW - gPW;
           nb[ri] = n * p.H;
           qq += 16;
           while (qq >= p.Q) {
@@ -352,10 +389,10 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         }
       }
       int kk = kb_begin * kBK + 8 * j;
-      int tap = kk / p.C;
-      int c = kk - tap * p.C;
-      int r = tap / p.S;
-      int s = tap - r * p.S;
+      int tap = kk / gC;
+      int c = kk - tap * gC;
+      int r = tap / gS;
+      int s = tap - r * gS;
       const int lag = min(2, stages - 1);
       int st = 0, st_lag = 0;  // ring slot being filled / being published
       uint32_t ph = 0;
@@ -363,7 +400,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         mbar_wait(empty0 + 8 * st, ph ^ 1);
         const uint32_t sa = smem_base + st * stage_bytes;
         const bool kval = kk < p.K;
-        const int dih = r * p.dh, diw = s * p.dw;
+        const int dih = r * gDH, diw = s * gDW;
 #pragma unroll
         for (int ri = 0; ri < 8; ++ri) {
           const int row = rg + 16 * ri;
@@ -372,7 +409,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           const int iw = iw0[ri] + diw;
           const bool ok = kval && rv[ri] && ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
           const __nv_bfloat16* src =
-              ok ? x + ((static_cast<int64_t>(nb[ri] + ih) * p.W + iw) * p.C + c) : x;
+              ok ? x + ((static_cast<int64_t>(nb[ri] + ih) * p.W + iw) * gC + c) : x;
           cp_async_16(dst, src, ok ? 16u : 0u);
         }
         cp_async_commit();
@@ -388,9 +425,9 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         }
         kk += kBK;
         c += kBK;
-        while (c >= p.C) {
-          c -= p.C;
-          if (++s == p.S) {
+        while (c >= gC) {
+          c -= gC;
+          if (++s == gS) {
             s = 0;
             ++r;
           }

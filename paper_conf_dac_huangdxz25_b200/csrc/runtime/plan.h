@@ -32,11 +32,13 @@ struct CatalogEntry {
   int32_t layout;
 };
 
+int32_t num_kernels();                 // generic + specialised
 const CatalogEntry& catalog(int32_t id);
 int64_t category_key(int32_t kernel_id);
+bool is_spec_kernel(int32_t kernel_id);  // a per-problem specialised conv solution
 
 bool is_applicable(int32_t kernel_id, const Problem& p, std::string* why = nullptr);
-int32_t static_choice(const Problem& p);
+int32_t static_choice(const Problem& p, int32_t catalog_mode = 0);
 
 // Validate the graph and extract problems.  Returns PASK_OK or an error with *err set.
 int extract_problems(const pask_graph* g, std::vector<Problem>* out, std::string* err);

@@ -20,7 +20,7 @@ OP_LAYOUT, OP_CONV2D, OP_GEMM, OP_POOL, OP_SOFTMAX, OP_LAYERNORM = range(6)
 ACT = {"none": 0, "relu": 1, "relu6": 2, "gelu": 3, "tanh": 4}
 K_LAYOUT, K_CONV_IGEMM, K_CONV_1X1, K_CONV_DW, K_POOL, K_POOL_GAVG, K_GEMM, K_SOFTMAX, \
     K_LAYERNORM = range(9)
-NUM_KERNELS = 9
+NUM_KERNELS = 9          # generic catalog (PASK_NUM_KERNELS); num_kernels() adds the specialisations
 HOW = {0: "direct", 1: "reused", 2: "loaded"}
 
 
@@ -56,7 +56,8 @@ class Graph(C.Structure):
 class Config(C.Structure):
     _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
                 ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
-                ("packaging", C.c_int32), ("interleave", C.c_int32), ("graph", C.c_int32)]
+                ("packaging", C.c_int32), ("interleave", C.c_int32), ("graph", C.c_int32),
+                ("catalog", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -141,8 +142,14 @@ def kernel_name(k):
 
 
 def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,
-           interleave=0, graph=0):
-    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph)
+           interleave=0, graph=0, catalog=0):
+    return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph,
+                  catalog)
+
+
+def num_kernels():
+    """Generic + specialised catalog size (pask_num_kernels)."""
+    return lib().pask_num_kernels()
 
 
 def plan(graph: Graph, cfg: Config | None = None):

@@ -29,6 +29,9 @@ SCHEMES = {
     "pask_r": dict(search=1),                         # PaSK-R: naive (exhaustive-order) search
     "reactive": dict(proactive=0, reuse=0),           # Baseline analog: lazy load at first launch
     "reactive_reuse": dict(proactive=0),              # reuse without the proactive loader
+    # tuned library (per-problem specialised conv solutions)
+    "baseline_tuned": dict(catalog=1, proactive=0, reuse=0),  # the paper's Baseline
+    "pask_tuned": dict(catalog=1),                    # PASK over the tuned library
 }
 
 
@@ -53,7 +56,7 @@ def child(model, scheme, batch=1):
     t1 = time.perf_counter_ns()
     st = ctx.stats()
     tl = {}
-    for k in range(P.NUM_KERNELS):
+    for k in range(P.num_kernels()):
         ld, rd, lb = ctx.kernel_timeline(k)
         if ld:
             tl[P.kernel_name(k)[5:]] = [round(lb / 1e3), round(ld / 1e3), round(rd / 1e3)]

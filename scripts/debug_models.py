@@ -19,7 +19,7 @@ for name in sys.argv[1:]:
     errs = teacher_forced_errors(dm, spec, x)
     st = ctx.stats()
     print(f"== {name}: infer+sync {1e3*(t1-t0):.1f} ms  stats {st}")
-    for k in range(P.NUM_KERNELS):
+    for k in range(P.num_kernels()):
         ld, rd, lb = ctx.kernel_timeline(k)
         if ld:
             print(f"  load {P.kernel_name(k):16s} load {ld/1e3:8.1f} us  ready@ {rd/1e3:8.1f} us  lib {lb/1e3:8.1f} us")

@@ -73,7 +73,8 @@ def test_struct_layouts_match_header(tmp_path):
             assert int(got[f"{cname}.{f}"]) == getattr(py, f).offset, (cname, f)
 
 
-CFGS = [dict(), dict(search=1), dict(reuse=0), dict(milestone=5), dict(milestone=1000)]
+CFGS = [dict(), dict(search=1), dict(reuse=0), dict(milestone=5), dict(milestone=1000),
+        dict(catalog=1), dict(catalog=1, reuse=0), dict(catalog=1, search=1)]
 
 
 @pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"])
@@ -86,7 +87,8 @@ def test_planner_matches_oracle_on_models(name):
         got, st = P.plan(dm.graph, cfg)
         exp = OP.execution_plan(probs, reuse=bool(cfg.reuse),
                                 search="naive" if cfg.search else "categorical",
-                                milestone=cfg.milestone)
+                                milestone=cfg.milestone,
+                                catalog="tuned" if cfg.catalog else "generic")
         assert [tuple(b) for b in got] == [tuple(b) for b in exp["bindings"]], kw
         assert (st["queries"], st["hits"], st["lookups"]) == \
             (exp["queries"], exp["hits"], exp["lookups"])
@@ -163,8 +165,8 @@ def test_unsupported_and_invalid_fail_loudly():
 
 def test_catalog_introspection_and_workspace():
     lib = P.lib()
-    assert lib.pask_num_kernels() == P.NUM_KERNELS
-    assert [P.kernel_name(k) for k in range(P.NUM_KERNELS)] == OP.KERNEL_NAMES
+    assert lib.pask_num_kernels() == len(OP.KERNEL_NAMES) == P.NUM_KERNELS + len(OP.SPECS)
+    assert [P.kernel_name(k) for k in range(P.num_kernels())] == OP.KERNEL_NAMES
     assert P.kernel_name(99) == ""
     spec, _ = build_model("resnet50")
     assert P.workspace_bytes(DeviceModel(spec, alloc=False).graph) == 0

@@ -28,7 +28,7 @@ def test_model_layers_teacher_forced(name):
     st = ctx.stats()
     assert st["kernels_loaded"] == len(o["loaded"])
     assert st["code_objects_loaded"] == len(o["loaded"])   # packaging 0: one object per kernel
-    loaded = {k for k in range(P.NUM_KERNELS) if ctx.kernel_is_loaded(k)}
+    loaded = {k for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k)}
     assert loaded == set(o["loaded"])
     assert len(loaded) <= 8
     ctx.close()
@@ -60,6 +60,27 @@ def test_graph_replay_bitwise(name):
     for a, n in zip(ref, spec["outputs"]):
         np.testing.assert_array_equal(a, dm.read_raw(n))
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "mobilenet_v2"])
+def test_tuned_catalog_specialised_kernels(name):
+    """The per-problem specialised solutions (tuned catalog, Baseline scheme):
+    every layer within tolerance, the loaded set = the plan oracle's, and every
+    layer's output bitwise equal to the generic kernels' (same tiling and
+    reduction order: a substitution never changes results)."""
+    spec, x = build_model(name)
+    dm, ctx, plan = run_model(spec, x, cfg=P.config(catalog=1, reuse=0, proactive=0))
+    errs = teacher_forced_errors(dm, spec, x)
+    assert max(e for _, _, e in errs) <= TOL
+    o = OP.execution_plan(OP.problems_from_spec(spec), reuse=False, catalog="tuned")
+    assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
+    assert {k for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k)} == set(o["loaded"])
+    tuned = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
+    ctx.close()
+    dm2, ctx2, _ = run_model(spec, x)
+    for L in spec["layers"]:
+        np.testing.assert_array_equal(tuned[L["out"]], dm2.read_raw(L["out"]))
+    ctx2.close()
 
 
 @pytest.mark.parametrize("packaging", [0, 1])

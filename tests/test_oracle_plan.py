@@ -177,3 +177,26 @@ def test_bruteforce_small_catalog_trace():
             stamp[got] = t
             assert pl["bindings"][i][2] == got
         assert (pl["queries"], pl["hits"], pl["lookups"]) == (q, h, lk)
+
+
+def test_tuned_catalog_covers_every_config_conv_and_plans():
+    """The tuned catalog holds exactly one specialisation per distinct dense-conv
+    (R, S, stride, pad, dilation, C) of configs C1-C3; with it the reactive
+    Baseline loads one conv kernel per such problem (ResNet-50: 17 + layout,
+    pool, gavg, FC, softmax = 22), while reuse cannot help (specialisations are
+    applicable only to their own shape)."""
+    combos = set()
+    for name in ("tiny_cnn", "resnet50", "mobilenet_v2"):
+        spec, _ = build_model(name)
+        for p in P.problems_from_spec(spec):
+            if p["op"] == P.CONV:
+                combos.add((p["r"], p["s"], p["stride_h"], p["pad_h"], p["dil_h"], p["c"]))
+    assert combos == set(P.SPECS) and len(P.SPECS) == 32
+    spec, _ = build_model("resnet50")
+    probs = P.problems_from_spec(spec)
+    base = P.execution_plan(probs, reuse=False, catalog="tuned")
+    assert len(base["loaded"]) == 22
+    pask = P.execution_plan(probs, catalog="tuned")
+    assert len(pask["loaded"]) == 21 and pask["hits"] == 1      # only gavg -> pool
+    for (i, want, bound, how, lk) in pask["bindings"]:
+        assert P.is_applicable(bound, probs[i])
