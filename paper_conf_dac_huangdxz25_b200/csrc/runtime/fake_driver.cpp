@@ -1,0 +1,202 @@
+// Test-only fake CUDA driver (include/pask_testing.h): exercises the loader /
+// issuer host logic without a GPU.  Handles are small integers disguised as
+// pointers; a CUfunction encodes its catalog kernel id (found from the name).
+#include <stdint.h>
+#include <string.h>
+
+#include <chrono>
+#include <mutex>
+#include <thread>
+#include <vector>
+
+#include "../../../include/pask_testing.h"
+#include "driver.h"
+#include "plan.h"
+
+#define PASK_API extern "C" __attribute__((visibility("default")))
+
+namespace pask {
+namespace {
+
+std::mutex g_mu;
+int g_load_us = 0;
+int g_fail_kernel = -1;
+std::vector<int32_t> g_ids, g_kinds;
+bool g_loaded[PASK_MAX_KERNELS] = {};
+
+int32_t kernel_of_name(const char* name) {
+  for (int32_t k = 0; k < num_kernels(); ++k)
+    if (strcmp(catalog(k).name, name) == 0) return k;
+  return -1;
+}
+void sleep_us(int us) {
+  if (us > 0) std::this_thread::sleep_for(std::chrono::microseconds(us));
+}
+void log_event(int32_t id, int32_t kind) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_ids.push_back(id);
+  g_kinds.push_back(kind);
+}
+template <class T>
+T fake_handle(uintptr_t v) {
+  return reinterpret_cast<T>(v);
+}
+constexpr uintptr_t kFnBase = 0x1000;
+
+CUresult f_ok_init(unsigned int) { return CUDA_SUCCESS; }
+CUresult f_err_name(CUresult r, const char** s) {
+  *s = r == CUDA_SUCCESS ? "CUDA_SUCCESS" : (r == CUDA_ERROR_INVALID_IMAGE ? "CUDA_ERROR_INVALID_IMAGE" : "CUDA_ERROR_FAKE");
+  return CUDA_SUCCESS;
+}
+CUresult f_dev_get(CUdevice* d, int o) {
+  *d = o;
+  return CUDA_SUCCESS;
+}
+CUresult f_ctx_get(CUcontext* c) {
+  *c = fake_handle<CUcontext>(0x10);
+  return CUDA_SUCCESS;
+}
+CUresult f_ctx_set(CUcontext) { return CUDA_SUCCESS; }
+CUresult f_lib_load(CUlibrary* lib, const void*, CUjit_option*, void**, unsigned int, CUlibraryOption*, void**,
+                    unsigned int) {
+  sleep_us(g_load_us);
+  *lib = fake_handle<CUlibrary>(0x20);
+  return CUDA_SUCCESS;
+}
+CUresult f_lib_unload(CUlibrary) { return CUDA_SUCCESS; }
+CUresult f_lib_get_kernel(CUkernel* k, CUlibrary, const char* name) {
+  const int32_t id = kernel_of_name(name);
+  if (id < 0) return CUDA_ERROR_NOT_FOUND;
+  *k = fake_handle<CUkernel>(kFnBase + id);
+  return CUDA_SUCCESS;
+}
+CUresult f_kernel_get_fn(CUfunction* f, CUkernel k) {
+  const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(k) - kFnBase);
+  sleep_us(g_load_us);
+  if (id == g_fail_kernel) return CUDA_ERROR_INVALID_IMAGE;
+  *f = fake_handle<CUfunction>(kFnBase + id);
+  return CUDA_SUCCESS;
+}
+CUresult f_func_load(CUfunction f) {
+  const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (id >= 0 && id < PASK_MAX_KERNELS) g_loaded[id] = true;
+  }
+  log_event(id, 0);
+  return CUDA_SUCCESS;
+}
+CUresult f_func_is_loaded(CUfunctionLoadingState* s, CUfunction f) {
+  const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
+  std::lock_guard<std::mutex> lk(g_mu);
+  *s = (id >= 0 && id < PASK_MAX_KERNELS && g_loaded[id]) ? CU_FUNCTION_LOADING_STATE_LOADED
+                                                          : CU_FUNCTION_LOADING_STATE_UNLOADED;
+  return CUDA_SUCCESS;
+}
+CUresult f_func_set_attr(CUfunction, CUfunction_attribute, int) { return CUDA_SUCCESS; }
+CUresult f_launch(const CUlaunchConfig*, CUfunction f, void**, void**) {
+  const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
+  bool loaded;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    loaded = id >= 0 && id < PASK_MAX_KERNELS && g_loaded[id];
+  }
+  log_event(id, loaded ? 1 : 2);
+  return CUDA_SUCCESS;
+}
+CUresult f_tmap_tiled(CUtensorMap* m, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
+                      const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                      CUtensorMapL2promotion, CUtensorMapFloatOOBfill) {
+  memset(m, 0, sizeof(*m));
+  return CUDA_SUCCESS;
+}
+CUresult f_tmap_im2col(CUtensorMap* m, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
+                       const int*, const int*, cuuint32_t, cuuint32_t, const cuuint32_t*, CUtensorMapInterleave,
+                       CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill) {
+  memset(m, 0, sizeof(*m));
+  return CUDA_SUCCESS;
+}
+CUresult f_event_create(CUevent* e, unsigned int) {
+  *e = fake_handle<CUevent>(0x30);
+  return CUDA_SUCCESS;
+}
+CUresult f_event_destroy(CUevent) { return CUDA_SUCCESS; }
+CUresult f_event_record(CUevent, CUstream) { return CUDA_SUCCESS; }
+CUresult f_event_sync(CUevent) { return CUDA_SUCCESS; }
+CUresult f_event_elapsed(float* ms, CUevent, CUevent) {
+  *ms = 0.f;
+  return CUDA_SUCCESS;
+}
+CUresult f_h2d(CUdeviceptr, const void*, size_t, CUstream) { return CUDA_SUCCESS; }
+CUresult f_d2h(void*, CUdeviceptr, size_t, CUstream) { return CUDA_SUCCESS; }
+CUresult f_stream_sync(CUstream) { return CUDA_SUCCESS; }
+CUresult f_stream_create(CUstream* s, unsigned int) {
+  *s = fake_handle<CUstream>(0x40);
+  return CUDA_SUCCESS;
+}
+CUresult f_stream_destroy(CUstream) { return CUDA_SUCCESS; }
+CUresult f_begin_capture(CUstream, CUstreamCaptureMode) { return CUDA_ERROR_NOT_SUPPORTED; }
+
+Driver make_fake() {
+  Driver d;
+  d.cuInit = f_ok_init;
+  d.cuGetErrorName = f_err_name;
+  d.cuDeviceGet = f_dev_get;
+  d.cuCtxGetCurrent = f_ctx_get;
+  d.cuCtxSetCurrent = f_ctx_set;
+  d.cuLibraryLoadData = f_lib_load;
+  d.cuLibraryUnload = f_lib_unload;
+  d.cuLibraryGetKernel = f_lib_get_kernel;
+  d.cuKernelGetFunction = f_kernel_get_fn;
+  d.cuFuncLoad = f_func_load;
+  d.cuFuncIsLoaded = f_func_is_loaded;
+  d.cuFuncSetAttribute = f_func_set_attr;
+  d.cuLaunchKernelEx = f_launch;
+  d.cuTensorMapEncodeTiled = f_tmap_tiled;
+  d.cuTensorMapEncodeIm2col = f_tmap_im2col;
+  d.cuEventCreate = f_event_create;
+  d.cuEventDestroy = f_event_destroy;
+  d.cuEventRecord = f_event_record;
+  d.cuEventSynchronize = f_event_sync;
+  d.cuEventElapsedTime = f_event_elapsed;
+  d.cuMemcpyHtoDAsync = f_h2d;
+  d.cuMemcpyDtoHAsync = f_d2h;
+  d.cuStreamSynchronize = f_stream_sync;
+  d.cuStreamCreate = f_stream_create;
+  d.cuStreamDestroy = f_stream_destroy;
+  d.cuStreamBeginCapture = f_begin_capture;
+  d.ok = true;
+  return d;
+}
+Driver g_fake;
+
+}  // namespace
+}  // namespace pask
+
+PASK_API int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail_kernel) {
+  using namespace pask;
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_load_us = load_us;
+  g_fail_kernel = fail_kernel;
+  g_ids.clear();
+  g_kinds.clear();
+  memset(g_loaded, 0, sizeof(g_loaded));
+  if (enable) {
+    g_fake = make_fake();
+    driver_override(&g_fake);
+  } else {
+    driver_override(nullptr);
+  }
+  return 0;
+}
+
+PASK_API int32_t pask_test_fake_log(int32_t* out, int32_t* kinds, int32_t cap) {
+  using namespace pask;
+  std::lock_guard<std::mutex> lk(g_mu);
+  const int32_t n = static_cast<int32_t>(g_ids.size());
+  for (int32_t i = 0; i < n && i < cap; ++i) {
+    if (out) out[i] = g_ids[i];
+    if (kinds) kinds[i] = g_kinds[i];
+  }
+  return n;
+}

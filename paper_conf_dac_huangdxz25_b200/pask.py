@@ -83,6 +83,7 @@ EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "
            "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
            "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name",
            "pask_kernel_timeline", "pask_node_times"]
+TEST_EXPORTS = ["pask_test_fake_driver", "pask_test_fake_log"]   # include/pask_testing.h
 
 _lib = None
 
@@ -114,6 +115,8 @@ def lib():
                                            C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
         "pask_node_times": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int32]),
         "pask_last_error": (C.c_char_p, []),
+        "pask_test_fake_driver": (C.c_int, [C.c_int32, C.c_int32, C.c_int32]),
+        "pask_test_fake_log": (C.c_int32, [C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.c_int32]),
         "pask_num_kernels": (C.c_int32, []),
         "pask_kernel_name": (C.c_char_p, [C.c_int32]),
     }
@@ -145,6 +148,19 @@ def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, pac
            interleave=0, graph=0, catalog=0):
     return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph,
                   catalog)
+
+
+def test_fake_driver(enable=True, load_us=0, fail_kernel=-1):
+    """Test-only (include/pask_testing.h): route new contexts to the fake driver."""
+    _check(lib().pask_test_fake_driver(1 if enable else 0, load_us, fail_kernel))
+
+
+def test_fake_log(cap=4096):
+    """[(kernel_id, kind)], kind 0 = load completed, 1 = launch, 2 = launch before load."""
+    ids = (C.c_int32 * cap)()
+    kinds = (C.c_int32 * cap)()
+    n = lib().pask_test_fake_log(ids, kinds, cap)
+    return [(ids[i], kinds[i]) for i in range(min(n, cap))]
 
 
 def num_kernels():

@@ -26,6 +26,7 @@ from workloads.models import _Builder
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 HEADER = os.path.join(ROOT, "include", "pask.h")
+TEST_HEADER = os.path.join(ROOT, "include", "pask_testing.h")
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -33,14 +34,14 @@ def built():
     pbuild.build()
 
 
-def header_functions():
-    src = open(HEADER).read()
+def header_functions(path=HEADER):
+    src = open(path).read()
     return sorted(set(re.findall(r"^\s*(?:const\s+)?\w+\s*\*?\s*(pask_\w+)\s*\(", src, re.M)))
 
 
 def test_exports_every_declared_symbol():
-    names = header_functions()
-    assert len(names) >= 15
+    names = header_functions() + header_functions(TEST_HEADER)
+    assert len(names) >= 17
     out = subprocess.run(["nm", "-D", "--defined-only", P.LIB_PATH], capture_output=True,
                          text=True).stdout
     exported = set(re.findall(r" T (pask_\w+)", out))
@@ -48,7 +49,7 @@ def test_exports_every_declared_symbol():
     lib = P.lib()
     for n in names:
         assert hasattr(lib, n)
-    assert set(P.EXPORTS) == set(names)
+    assert set(P.EXPORTS) | set(P.TEST_EXPORTS) == set(names)
     assert lib.pask_version() >= 100
 
 

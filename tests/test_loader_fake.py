@@ -1,0 +1,130 @@
+"""T2: loader / issuer host logic on CPU through the fake driver
+(include/pask_testing.h).  No GPU: every driver call goes to an in-library
+fake that sleeps on loads and records loads and launches.
+
+Checks, for every proactive / interleave / packaging / reuse mode:
+* uploads happen once per planned kernel, in first-use order;
+* no launch precedes the completed load of its kernel;
+* the launch sequence is the plan's bound kernel of each node, in node order;
+* a failed load propagates as PASK_ECUDA naming the kernel (no fallback);
+* nothing deadlocks (pytest-timeout), including destroy with pending loads.
+"""
+import pytest
+
+from oracle import plan as OP
+from paper_conf_dac_huangdxz25_b200 import build as pbuild
+from paper_conf_dac_huangdxz25_b200 import pask as P
+from paper_conf_dac_huangdxz25_b200.model import DeviceModel
+from workloads import build_model
+
+pytestmark = pytest.mark.timeout(120)
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    pbuild.build()
+    yield
+    P.test_fake_driver(False)
+
+
+MODES = [
+    dict(proactive=2), dict(proactive=1), dict(proactive=1, interleave=1), dict(proactive=0),
+    dict(proactive=2, packaging=1), dict(proactive=2, reuse=0), dict(proactive=1, search=1),
+    dict(proactive=0, reuse=0, catalog=1), dict(proactive=2, catalog=1),
+]
+
+
+@pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "bert_base"])
+@pytest.mark.parametrize("mode", MODES, ids=[str(m) for m in MODES])
+def test_load_order_and_launch_safety(name, mode):
+    spec, _ = build_model(name)
+    dm = DeviceModel(spec, alloc=False)
+    P.test_fake_driver(True, load_us=300)
+    ctx = P.Context(0, P.config(**mode))
+    plan = ctx.load_model(dm.graph)
+    for _ in range(2):                      # cold, then hot
+        ctx.infer(0)
+        ctx.sync()
+    st = ctx.stats()
+    ctx.close()
+    log = P.test_fake_log()
+    loads = [k for k, kind in log if kind == 0]
+    launches = [(k, kind) for k, kind in log if kind != 0]
+    exp = OP.execution_plan(OP.problems_from_spec(spec), reuse=bool(mode.get("reuse", 1)),
+                            search="naive" if mode.get("search") else "categorical",
+                            catalog="tuned" if mode.get("catalog") else "generic")
+    assert loads == exp["loaded"]                                   # once each, first-use order
+    assert all(kind == 1 for _, kind in launches)                   # never before its load
+    bound = [b[2] for b in plan]
+    assert [k for k, _ in launches] == bound + bound                # node order, 2 inferences
+    assert st["kernels_loaded"] == len(exp["loaded"])
+    assert st["launches"] == 2 * len(bound)
+    if mode.get("proactive", 2) == 2:
+        assert st["load_exposed_ns"] == 0                           # all uploads inside load_model
+
+
+@pytest.mark.parametrize("mode", [dict(proactive=2), dict(proactive=1), dict(proactive=0),
+                                  dict(proactive=1, interleave=1)])
+def test_failed_load_propagates(mode):
+    spec, _ = build_model("resnet50")
+    dm = DeviceModel(spec, alloc=False)
+    P.test_fake_driver(True, load_us=100, fail_kernel=P.K_CONV_IGEMM)
+    ctx = P.Context(0, P.config(**mode))
+    with pytest.raises(P.PaskError) as ei:
+        ctx.load_model(dm.graph)
+        ctx.infer(0)
+    assert ei.value.code == P.ECUDA
+    assert "pask_conv_igemm" in str(ei.value) and "CUDA_ERROR_INVALID_IMAGE" in str(ei.value)
+    ctx.close()
+    launched = [k for k, kind in P.test_fake_log() if kind != 0]
+    assert P.K_CONV_IGEMM not in launched
+    # only the layout node (before the first conv) may have been issued
+    assert set(launched) <= {P.K_LAYOUT}
+
+
+def test_destroy_with_pending_loads_and_reuse_across_models():
+    P.test_fake_driver(True, load_us=2000)
+    spec, _ = build_model("resnet50")
+    dm = DeviceModel(spec, alloc=False)
+    ctx = P.Context(0, P.config(proactive=1))
+    ctx.load_model(dm.graph)
+    ctx.close()                              # joins the loader with loads still queued
+    # a second model in a fresh context after a first one: no stale state
+    P.test_fake_driver(True, load_us=0)
+    ctx = P.Context(0, P.config())
+    spec2, _ = build_model("mobilenet_v2")
+    ctx.load_model(DeviceModel(spec2, alloc=False).graph)
+    ctx.infer(0)
+    ctx.sync()
+    assert ctx.stats()["kernels_loaded"] == 6
+    ctx.close()
+
+
+def test_rebinding_inputs_relowers_without_reloading():
+    P.test_fake_driver(True, load_us=0)
+    spec, _ = build_model("tiny_cnn")
+    dm = DeviceModel(spec, alloc=False)
+    ctx = P.Context(0, P.config())
+    ctx.load_model(dm.graph)
+    ctx.infer(0)
+    ctx.infer(0, inputs=[1 << 22], outputs=[1 << 23])   # new buffers: parameters re-encoded
+    ctx.sync()
+    st = ctx.stats()
+    ctx.close()
+    assert st["kernels_loaded"] == 5 and st["launches"] == 14
+    assert sum(1 for _, kind in P.test_fake_log() if kind == 0) == 5
+
+
+def test_state_errors():
+    P.test_fake_driver(True)
+    ctx = P.Context(0, P.config())
+    with pytest.raises(P.PaskError) as ei:
+        ctx.infer(0)
+    assert ei.value.code == P.ESTATE
+    spec, _ = build_model("tiny_cnn")
+    dm = DeviceModel(spec, alloc=False)
+    ctx.load_model(dm.graph)
+    with pytest.raises(P.PaskError) as ei:
+        ctx.load_model(dm.graph)             # one model per context
+    assert ei.value.code == P.ESTATE
+    ctx.close()
