@@ -231,6 +231,8 @@ typedef struct {
   uint64_t infer_entry_ns;     /*   last planned kernel uploaded, first pask_infer */
   uint64_t first_launch_ns;    /*   entry, its first and last launch              */
   uint64_t last_launch_ns;
+  uint64_t encode_begin_ns;    /* launch-parameter encoding window, ns after      */
+  uint64_t encode_end_ns;      /*   pask_load_model entry                         */
 } pask_stats_t;
 
 /* Library version (PASK_VERSION). */
@@ -279,6 +281,19 @@ int pask_infer(pask_ctx *ctx, void *const *inputs, void *const *outputs, void *c
  * recommended; sizes follow the tensors' dims and dtype. */
 int pask_infer_host(pask_ctx *ctx, const void *const *host_inputs, void *const *host_outputs,
                     void *cuda_stream);
+
+/* Idle-interval loading (§VI "Loading desired solutions"): upload
+ * the solutions Algorithm 1 skipped and rebind those nodes to them.
+ *   target_catalog < 0: the model's own catalog -- every reused node goes back
+ *                       to its s*_i;
+ *   target_catalog 0/1: re-run the static choice under that catalog (1 = the
+ *                       tuned per-problem solutions) and bind every node whose
+ *                       choice differs from its current kernel.
+ * Synchronous and meant for the gap between requests: it first waits for the
+ * in-flight inference (uploads wait for running GPU work, D3).
+ * Results stay within tolerance; a graph captured for hot replay is re-captured.
+ * *promoted (may be NULL) = number of nodes rebound. */
+int pask_promote(pask_ctx *ctx, int32_t target_catalog, int32_t *promoted);
 
 /* Wait for the last issued inference and finalise its timing statistics
  * (gpu_span_ns; cold_wall_ns after the first inference). */

@@ -14,11 +14,12 @@
 //   conv: m = output pixel (n, p, q), n = output channel, k = (r, s, c) in KRSC order,
 //         A[m][k] = X[n, p*sh - ph + r*dh, q*sw - pw + s*dw, c] (0 outside)
 //
-// Structure (192 threads, one 128 x BN output tile per CTA, or per cluster):
-//   warps 0-3 : bias -> smem; A_GATHER: implicit im2col producer (cp.async,
-//               16 B per lane, SWIZZLE_128B placement); then the epilogue
-//   warp 4    : TMA producer (B always, A in A_TMA mode, the residual tile)
-//   warp 5    : TMEM allocator + single-thread tcgen05.mma issuer
+// Structure (320 threads, one 128 x BN output tile per CTA, or per cluster):
+//   warps 0-7 : bias -> smem; A_GATHER: implicit im2col producer (cp.async,
+//               16 B per lane, SWIZZLE_128B placement); then the epilogue, two
+//               warps per TMEM lane quarter (alternate 16-column chunks)
+//   warp 8    : TMA producer (B always, A in A_TMA mode, the residual tile)
+//   warp 9    : TMEM allocator + single-thread tcgen05.mma issuer
 //   smem      : ring of `stages` x {A 128x64, B BNx64} bf16 with full/empty
 //               mbarriers; residual/output staging tile; bias vector
 //   epilogue  : TMEM -> registers -> (+bias, +residual from smem, act) -> bf16
@@ -40,7 +41,9 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// Activation over 16 values: one loop per activation kind (compact SASS).
+// Activation over 16 values: ReLU / ReLU6 inline; GELU / tanh (transformer
+// GEMMs) through one out-of-line routine to keep the code object small.
+__device__ __noinline__ float act_slow(float v, int act) { return apply_act(v, act); }
 __device__ __forceinline__ void act16(float (&v)[16], int act) {
   if (act == 1) {
 #pragma unroll
@@ -48,79 +51,72 @@ __device__ __forceinline__ void act16(float (&v)[16], int act) {
   } else if (act == 2) {
 #pragma unroll
     for (int i = 0; i < 16; ++i) v[i] = fminf(fmaxf(v[i], 0.f), 6.f);
-  } else if (act == 3) {
+  } else if (act >= 3) {
 #pragma unroll
-    for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i], 3);
-  } else if (act == 4) {
-#pragma unroll
-    for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i], 4);
+    for (int i = 0; i < 16; ++i) v[i] = act_slow(v[i], act);
   }
 }
 
-// Layout of the residual / output staging tile: column boxes of box_cols
-// (16/32/48/64) columns, each 128 rows x box_cols bf16; 64-wide boxes use the
-// TMA SWIZZLE_128B pattern (16 B chunk c of row r at chunk c ^ (r & 7)).
-__device__ __forceinline__ uint32_t ro_chunk(uint32_t ro, int box_cols, int row, int col) {
-  const int j = col / box_cols;
-  const int cc = (col - j * box_cols) >> 3;
-  const uint32_t base = ro + j * (128 * box_cols * 2) + row * (box_cols * 2);
-  return box_cols == 64 ? base + ((cc ^ (row & 7)) << 4) : base + (cc << 4);
+// Layout of the residual / output staging tile: column boxes of 2^lb (16/32/64)
+// columns, each 128 rows x 2^lb bf16; 64-wide boxes use the TMA SWIZZLE_128B
+// pattern (16 B chunk c of row r at chunk c ^ (r & 7)).  col is a multiple of 8.
+__device__ __forceinline__ uint32_t ro_addr(uint32_t ro, int lb, int row, int col) {
+  const int j = col >> lb;
+  const int cc = (col & ((1 << lb) - 1)) >> 3;
+  const uint32_t base = ro + (static_cast<uint32_t>(j * 128 + row) << (lb + 1));
+  return lb == 6 ? base + ((cc ^ (row & 7)) << 4) : base + (cc << 4);
 }
+// box width of the staged epilogue for an N tile of bn columns (power of two)
+__device__ __forceinline__ int box_log2(int bn) { return bn >= 64 ? 6 : (bn == 32 ? 5 : 4); }
 
-struct EpiCtx {
-  const float* s_bias;  // smem, bn floats (0 outside N)
-  uint32_t ro;          // smem staging tile (c_tma)
-  int box_cols;
-  int m0, n0, b;
-};
-
-// v = act(acc + bias + res) -> bf16 (RNE) for 16 columns of tile row `row`:
-// staged in smem for the TMA store (c_tma) or stored directly (unaligned output).
-__device__ __forceinline__ void epi16(const GemmParams& p, const EpiCtx& e, int row, int cb,
-                                      float (&v)[16]) {
+// v = act(acc + bias + res) -> bf16 (RNE) for 16 columns [cb, cb+16) of tile row
+// `row`: staged in smem for the TMA store (c_tma) or stored directly.
+__device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint32_t ro, int lb, int m0,
+                                      int n0, int b, int row, int cb, float (&v)[16]) {
 #pragma unroll
-  for (int i = 0; i < 16; ++i) v[i] += e.s_bias[cb + i];
-  const int m = e.m0 + row, n = e.n0 + cb;
-  const uint32_t a0 = ro_chunk(e.ro, e.box_cols, row, cb);
-  const uint32_t a1 = ro_chunk(e.ro, e.box_cols, row, cb + 8);
-  const bool in = m < p.M && n < p.N;
-  const int nv = min(16, p.N - n);
-  const int64_t base = p.off_c + static_cast<int64_t>(e.b) * p.stride_c + static_cast<int64_t>(m) * p.ldc + n;
-  if (p.res) {
-    float f[16];
-    if (p.c_tma) {
-      uint4 r0, r1;
-      asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r0.x), "=r"(r0.y), "=r"(r0.z), "=r"(r0.w) : "r"(a0));
-      asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r1.x), "=r"(r1.y), "=r"(r1.z), "=r"(r1.w) : "r"(a1));
+  for (int q4 = 0; q4 < 4; ++q4) {
+    const float4 bb = lds_f4(sbias + (cb + 4 * q4) * 4);  // broadcast
+    v[4 * q4] += bb.x;
+    v[4 * q4 + 1] += bb.y;
+    v[4 * q4 + 2] += bb.z;
+    v[4 * q4 + 3] += bb.w;
+  }
+  if (p.c_tma) {
+    const uint32_t a0 = ro_addr(ro, lb, row, cb);
+    const uint32_t a1 = ro_addr(ro, lb, row, cb + 8);
+    if (p.res) {
       float f0[8], f1[8];
-      unpack_bf16x8(r0, f0);
-      unpack_bf16x8(r1, f1);
+      unpack_bf16x8(lds_u4(a0), f0);
+      unpack_bf16x8(lds_u4(a1), f1);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        f[i] = f0[i];
-        f[8 + i] = f1[i];
+        v[i] += f0[i];
+        v[8 + i] += f1[i];
       }
-    } else {
-      const __nv_bfloat16* res = reinterpret_cast<const __nv_bfloat16*>(p.res);
-#pragma unroll
-      for (int i = 0; i < 16; ++i) f[i] = (in && i < nv) ? __bfloat162float(res[base + i]) : 0.f;
     }
-#pragma unroll
-    for (int i = 0; i < 16; ++i) v[i] += f[i];
+    act16(v, p.act);
+    sts_u4(a0, pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+           pack_bf16x2(v[6], v[7]));
+    sts_u4(a1, pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
+           pack_bf16x2(v[14], v[15]));
+    return;
   }
-  act16(v, p.act);
-  uint32_t pk[8];
-#pragma unroll
-  for (int i = 0; i < 8; ++i) pk[i] = pack_bf16x2(v[2 * i], v[2 * i + 1]);
-  if (p.c_tma) {
-    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a0), "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]) : "memory");
-    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a1), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]) : "memory");
-  } else if (in) {
-    unsigned short* o16 = reinterpret_cast<unsigned short*>(p.out) + base;
+  // unaligned output rows (e.g. N = 10): scalar stores, residual from global
+  const int m = m0 + row, n = n0 + cb;
+  if (m >= p.M || n >= p.N) return;
+  const int nv = min(16, p.N - n);
+  const int64_t base = p.off_c + static_cast<int64_t>(b) * p.stride_c + static_cast<int64_t>(m) * p.ldc + n;
+  if (p.res) {
+    const __nv_bfloat16* res = reinterpret_cast<const __nv_bfloat16*>(p.res);
 #pragma unroll
     for (int i = 0; i < 16; ++i)
-      if (i < nv) o16[i] = static_cast<unsigned short>((pk[i >> 1] >> (16 * (i & 1))) & 0xFFFFu);
+      if (i < nv) v[i] += __bfloat162float(res[base + i]);
   }
+  act16(v, p.act);
+  __nv_bfloat16* o = reinterpret_cast<__nv_bfloat16*>(p.out) + base;
+#pragma unroll
+  for (int i = 0; i < 16; ++i)
+    if (i < nv) o[i] = __float2bfloat16_rn(v[i]);
 }
 
 // Geometry policy of the contraction body.  DynGeo reads filter size, stride,
@@ -201,46 +197,61 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int kb_end = static_cast<int>((static_cast<int64_t>(split + 1) * p.num_kb) / splits);
   const int nk = kb_end - kb_begin;  // >= 1 (host guarantees num_kb >= splits)
   const int m0 = mt * kBM, n0 = nt * bn;
-  const int box_cols = bn < 64 ? bn : 64;
+  const int lb = box_log2(bn);
+  const int box_cols = 1 << lb;
   const int rows_per = p.rows_per;
   const int r0 = splits > 1 ? static_cast<int>(cluster_ctarank()) * rows_per : 0;
+  // rows of this tile inside the output, and of this rank's slice (split-K)
+  const int valid_rows = min(kBM, p.M - m0);
+  const int slice_rows = max(0, min(rows_per, valid_rows - r0));
   const bool res_tma = p.c_tma && p.res != nullptr;
   unsigned long long* trace =
       p.trace ? p.trace + 8ull * (blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) : nullptr;
-  if (trace && t == 0) trace[0] = globaltimer();
+  // debug phase stamps: [0] start [1] prologue done [2] producer past griddepcontrol.wait
+  // [3] first k-block landed [4] first accumulator chunk in registers (or split-K
+  // partials pushed) [5] accumulator ready [6] epilogue math done [7] tile stored
+  auto stamp = [&]() -> unsigned long long {
+    if (p.trace_clock) {
+      unsigned long long c;
+      asm volatile("mov.u64 %0, %%clock64;" : "=l"(c));
+      return c;
+    }
+    return globaltimer();
+  };
+  if (trace && t == 0) trace[0] = stamp();
 
   // ---------------- prologue (overlaps the previous kernel under PDL)
   if (t == 0) {
     for (int s = 0; s < stages; ++s) {
-      mbar_init(full0 + 8 * s, gather ? 129u : 1u);
+      mbar_init(full0 + 8 * s, gather ? kEpiThreads + 1u : 1u);
       mbar_init(empty0 + 8 * s, 1u);
     }
     mbar_init(accum_bar, 1u);
     mbar_init(res_bar, 1u);
     mbar_init(recv_bar, 1u);
-    if (splits > 1)  // the S-1 peers push rows_per x bn fp32 each into this CTA
-      mbar_arrive_expect_tx(recv_bar, static_cast<uint32_t>((splits - 1) * rows_per * bn * 4));
+    if (splits > 1)  // the S-1 peers push the valid rows of this rank's slice, bn fp32 each
+      mbar_arrive_expect_tx(recv_bar, static_cast<uint32_t>((splits - 1) * slice_rows * bn * 4));
     fence_barrier_init();
   }
-  if (warp == 4 && lane == 0) {
+  if (warp == kEpiWarps && lane == 0) {
     if (!gather) tma_prefetch_desc(&p.tmap_a);
     tma_prefetch_desc(&p.tmap_b);
     if (p.c_tma) tma_prefetch_desc(&p.tmap_c);
     if (res_tma) tma_prefetch_desc(&p.tmap_r);
   }
-  if (warp == 5) tmem_alloc(smem_u32(tmem_slot), p.tmem_cols);
+  if (warp == kEpiWarps + 1) tmem_alloc(smem_u32(tmem_slot), p.tmem_cols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   if (splits > 1) cluster_sync_all();  // peers' receive barriers are initialised
   const uint32_t tmem_base = *tmem_slot;
-  if (trace && t == 0) trace[1] = globaltimer();
+  if (trace && t == 0) trace[1] = stamp();
 
   pdl_launch_dependents();  // let the next layer's prologue start
   // griddepcontrol.wait is per role: weights (B, bias) do not depend on the
   // previous layer, so they are fetched before it; activations after it.
 
-  if (warp == 4) {
+  if (warp == kEpiWarps) {
     // ================= TMA producer
     if (lane == 0) {
       // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
@@ -276,8 +287,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         }
       }
       pdl_wait();  // activations / residual of this layer are complete and visible
-      if (trace) trace[2] = globaltimer();
-      if (res_tma) {  // residual rows [r0, r0 + rows_per) of the tile, consumed by the epilogue
+      if (trace) trace[2] = stamp();
+      if (res_tma && slice_rows > 0) {  // residual rows [r0, r0 + rows_per), read by the epilogue
         mbar_arrive_expect_tx(res_bar, static_cast<uint32_t>(rows_per * bn * 2));
 #pragma unroll 1
         for (int j = 0; j < bn / box_cols; ++j)
@@ -322,7 +333,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       }
     }
     __syncwarp();
-  } else if (warp == 5) {
+  } else if (warp == kEpiWarps + 1) {
     // ================= MMA issuer (one thread issues for the whole CTA)
     if (lane == 0) {
       int s = 0;
@@ -330,7 +341,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       for (int i = 0; i < nk; ++i) {
         mbar_wait(full0 + 8 * s, ph);
         tc_fence_after();
-        if (trace && i == 0) trace[3] = globaltimer();
+        if (trace && i == 0) trace[3] = stamp();
         const uint32_t sa = smem_base + s * stage_bytes;
         const uint32_t sb = sa + kABytes;
 #pragma unroll
@@ -350,22 +361,23 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         }
       }
       umma_commit(accum_bar);  // accumulator complete -> epilogue
-      if (trace) trace[4] = globaltimer();
     }
     __syncwarp();
   } else {
-    // ================= warps 0-3: bias, (gather), epilogue
+    // ================= warps 0-7: bias, (gather), epilogue
     if (t < bn) s_bias[t] = (p.bias != nullptr && n0 + t < p.N) ? __ldg(p.bias + n0 + t) : 0.f;
     pdl_wait();  // before reading this layer's activations (gather) or writing outputs
     if (kAllowGather && gather) {
-      // implicit im2col: lane t owns 16 B chunk j = t % 8 of rows rg + 16 * ri
+      // implicit im2col: thread t owns 16 B chunk j = t % 8 of rows rg + kGR * ri
+      constexpr int kGR = kEpiThreads / 8;  // rows per pass
+      constexpr int kGI = kBM / kGR;        // passes per 128-row tile
       const int j = t & 7;
       const int rg = t >> 3;
       const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x);
-      int ih0[8], iw0[8], nb[8];
-      bool rv[8];
+      int ih0[kGI], iw0[kGI], nb[kGI];
+      bool rv[kGI];
       {
-        // output pixel of row rg, then step 16 pixels per ri (no per-row divisions)
+        // output pixel of row rg, then step kGR pixels per ri (no per-row divisions)
         const int m = m0 + rg;
         const int pq = p.P * p.Q;
         int n = m / pq;
@@ -373,12 +385,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         int pp = rem / p.Q;
         int qq = rem - pp * p.Q;
 #pragma unroll
-        for (int ri = 0; ri < 8; ++ri) {
-          rv[ri] = (m + 16 * ri) < p.M;
+        for (int ri = 0; ri < kGI; ++ri) {
+          rv[ri] = (m + kGR * ri) < p.M;
           ih0[ri] = pp * gSH - gPH;
           iw0[ri] = qq * gSW - gPW;
           nb[ri] = n * p.H;
-          qq += 16;
+          qq += kGR;
           while (qq >= p.Q) {
             qq -= p.Q;
             if (++pp == p.P) {
@@ -402,8 +414,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const bool kval = kk < p.K;
         const int dih = r * gDH, diw = s * gDW;
 #pragma unroll
-        for (int ri = 0; ri < 8; ++ri) {
-          const int row = rg + 16 * ri;
+        for (int ri = 0; ri < kGI; ++ri) {
+          const int row = rg + kGR * ri;
           const uint32_t dst = sa + row * 128 + ((j ^ (row & 7)) << 4);
           const int ih = ih0[ri] + dih;
           const int iw = iw0[ri] + diw;
@@ -440,116 +452,133 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         if (++st_lag == stages) st_lag = 0;
       }
     }
-    named_bar_sync(1, 128);  // s_bias complete
+    named_bar_sync(1, kEpiThreads);  // s_bias complete
     mbar_wait(accum_bar, 0);
     tc_fence_after();
-    if (trace && t == 0) trace[5] = globaltimer();
+    if (trace && t == 0) trace[5] = stamp();
   }
 
-  // ---------------- epilogue
-  EpiCtx e{s_bias, ro, box_cols, m0, n0, b};
-  const uint32_t taddr = tmem_base + (static_cast<uint32_t>((warp & 3) * 32) << 16);
-  const int cpr = bn >> 4;  // 16-column chunks per row
-  if (splits > 1 && warp < 4) {
-    // push this split's fp32 rows to their owners' receive slot [my rank]
-    const int row = warp * 32 + lane;
-    const uint32_t owner = static_cast<uint32_t>(row / rows_per);
-    const uint32_t me = cluster_ctarank();
-    const uint32_t slot_row = me * rows_per + (row - owner * rows_per);
-    const uint32_t local = recv + slot_row * recv_pitch;
-    const uint32_t remote = mapa_cluster(local, owner);
-    const uint32_t rbar = mapa_cluster(recv_bar, owner);
-    for (int cb = 0; cb < bn; cb += 16) {
-      float v[16];
-      tmem_ld16(taddr + cb, v);
+  // ---------------- epilogue: warp w (0-7) reads TMEM lanes / tile rows
+  // 32*(w%4) .. +31 (the tcgen05.ld lane quarter of its warp) and the 16-column
+  // chunks c with c % 2 == w / 4.  Rows at or beyond M are never read or stored.
+  if (warp < kEpiWarps) {
+    const int quarter = warp & 3;
+    const int half = warp >> 2;
+    const int row = quarter * 32 + lane;
+    const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
+    const int cpr = bn >> 4;  // 16-column chunks per row
+    const uint32_t sbias = smem_u32(s_bias);
+    const bool warp_live = quarter * 32 < valid_rows;  // warp-uniform: tcgen05.ld is .sync.aligned
+    uint32_t r[16];
+    if (splits > 1) {
+      // push this split's fp32 partial rows to their owners' receive slot [my rank]
+      const uint32_t owner = static_cast<uint32_t>(row / rows_per);
+      const uint32_t me = cluster_ctarank();
+      const uint32_t slot_row = me * rows_per + (row - owner * rows_per);
+      const uint32_t local = recv + slot_row * recv_pitch;
+      const uint32_t remote = mapa_cluster(local, owner);
+      const uint32_t rbar = mapa_cluster(recv_bar, owner);
+      const bool live = row < valid_rows;
+      if (warp_live) {
+        int c = half;
+        if (c < cpr) {
+          tmem_ld16_issue(taddr + c * 16, r);
+          tmem_ld_wait(r);
+        }
+        for (; c < cpr; c += 2) {
+          uint32_t u[16];
 #pragma unroll
-      for (int q4 = 0; q4 < 4; ++q4) {
-        if (owner == me)
-          asm volatile("st.shared.v4.f32 [%0], {%1,%2,%3,%4};" ::"r"(local + (cb + 4 * q4) * 4),
-                       "f"(v[4 * q4]), "f"(v[4 * q4 + 1]), "f"(v[4 * q4 + 2]), "f"(v[4 * q4 + 3])
-                       : "memory");
-        else
-          st_async_f4(remote + (cb + 4 * q4) * 4, v[4 * q4], v[4 * q4 + 1], v[4 * q4 + 2], v[4 * q4 + 3],
-                      rbar);
+          for (int i = 0; i < 16; ++i) u[i] = r[i];
+          const bool more = c + 2 < cpr;
+          if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
+          if (live) {
+#pragma unroll
+            for (int q4 = 0; q4 < 4; ++q4) {
+              const uint32_t off = (c * 16 + 4 * q4) * 4;
+              const float x0 = __uint_as_float(u[4 * q4]), x1 = __uint_as_float(u[4 * q4 + 1]);
+              const float x2 = __uint_as_float(u[4 * q4 + 2]), x3 = __uint_as_float(u[4 * q4 + 3]);
+              if (owner == me)
+                sts_f4(local + off, x0, x1, x2, x3);
+              else
+                st_async_f4(remote + off, x0, x1, x2, x3, rbar);
+            }
+          }
+          if (more) tmem_ld_wait(r);
+        }
+      }
+      if (trace && t == 0) trace[4] = stamp();
+      named_bar_sync(1, kEpiThreads);  // own-slot rows visible to all epilogue threads
+      mbar_wait(recv_bar, 0);          // every peer's rows have landed
+      if (res_tma && slice_rows > 0) mbar_wait(res_bar, 0);
+    } else {
+      if (res_tma) mbar_wait(res_bar, 0);
+      if (warp_live && half < cpr) {
+        tmem_ld16_issue(taddr + half * 16, r);
+        tmem_ld_wait(r);
+        if (trace && t == 0) trace[4] = stamp();
       }
     }
-    named_bar_sync(1, 128);  // own-slot rows visible to all epilogue threads
-    mbar_wait(recv_bar, 0);  // every peer's rows have landed
-  }
-  if (warp < 4) {
-    if (res_tma) mbar_wait(res_bar, 0);
-    // items: (row, 16-column chunk).  splits == 1: thread t owns TMEM lane / row t.
-    // splits > 1: the 128 threads stride over this rank's rows_per x cpr items.
-    // items: (row, 16-column chunk).  splits == 1: thread t owns TMEM lane / row t
-    // and reads 32 columns per tcgen05.ld; splits > 1: the 128 threads stride
-    // over this rank's rows_per x cpr items and reduce the S receive slots.
-    const int n_items = splits == 1 ? cpr : (rows_per * cpr - t + 127) / 128;
-    float buf[32];
-    for (int k = 0; k < n_items; ++k) {
-      int row, cb;
+    // one epilogue loop (a single epi16 site keeps the code object small):
+    //   splits == 1: this warp's chunks c = half, half + 2, ..., TMEM reads software-
+    //                pipelined (chunk c + 2 in flight while c is processed);
+    //   splits  > 1: items (row, chunk) of this rank's slice, the S receive slots
+    //                summed in fixed rank order 0..S-1 (deterministic)
+    const int n_iter = splits == 1 ? (warp_live && half < cpr ? (cpr - half + 1) >> 1 : 0)
+                                   : max(0, (slice_rows * cpr - t + kEpiThreads - 1) / kEpiThreads);
+    for (int k = 0; k < n_iter; ++k) {
       float v[16];
+      int erow, cb;
+      bool more = false;
       if (splits == 1) {
-        row = t;
-        cb = k << 4;
-        const bool odd = (k & 1) != 0;
-        if (!odd) {
-          if (cb + 32 <= bn) {
-            tmem_ld32(taddr + cb, buf);  // warp-collective
-          } else {
-            float h[16];
-            tmem_ld16(taddr + cb, h);
+        const int c = half + 2 * k;
+        erow = row;
+        cb = c * 16;
 #pragma unroll
-            for (int i = 0; i < 16; ++i) buf[i] = h[i];
-          }
-        }
-#pragma unroll
-        for (int i = 0; i < 16; ++i) v[i] = odd ? buf[16 + i] : buf[i];
+        for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+        more = c + 2 < cpr;
+        if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
       } else {
-        const int it = t + 128 * k;
-        const int lr = it / cpr;  // row within this rank's slice
-        row = r0 + lr;
+        const int it = t + k * kEpiThreads;
+        const int lr = it / cpr;
+        erow = r0 + lr;
         cb = (it - lr * cpr) << 4;
         const uint32_t src = recv + lr * recv_pitch + cb * 4;
 #pragma unroll
         for (int i = 0; i < 16; ++i) v[i] = 0.f;
-        for (int sp = 0; sp < splits; ++sp) {  // fixed rank order: deterministic
+        for (int sp = 0; sp < splits; ++sp) {
           const uint32_t a = src + sp * rows_per * recv_pitch;
-          float4 f[4];
-#pragma unroll
-          for (int q4 = 0; q4 < 4; ++q4)
-            asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
-                         : "=f"(f[q4].x), "=f"(f[q4].y), "=f"(f[q4].z), "=f"(f[q4].w)
-                         : "r"(a + 16 * q4));
 #pragma unroll
           for (int q4 = 0; q4 < 4; ++q4) {
-            v[4 * q4] += f[q4].x;
-            v[4 * q4 + 1] += f[q4].y;
-            v[4 * q4 + 2] += f[q4].z;
-            v[4 * q4 + 3] += f[q4].w;
+            const float4 f = lds_f4(a + 16 * q4);
+            v[4 * q4] += f.x;
+            v[4 * q4 + 1] += f.y;
+            v[4 * q4 + 2] += f.z;
+            v[4 * q4 + 3] += f.w;
           }
         }
       }
-      epi16(p, e, row, cb, v);
+      if (erow < valid_rows) epi16(p, sbias, ro, lb, m0, n0, b, erow, cb, v);
+      if (more) tmem_ld_wait(r);
     }
-  }
-  if (trace && t == 0) trace[6] = globaltimer();
-  if (p.c_tma && warp < 4) {
-    fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
-    named_bar_sync(1, 128);
-    if (t == 0) {
+    if (trace && t == 0) trace[6] = stamp();
+    if (p.c_tma) {
+      fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
+      named_bar_sync(1, kEpiThreads);
+      if (t == 0 && slice_rows > 0) {
 #pragma unroll 1
-      for (int j = 0; j < bn / box_cols; ++j)
-        tma_store_3d(&p.tmap_c, ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), n0 + j * box_cols,
-                     m0 + r0, b);
-      tma_store_commit_and_wait_read();
+        for (int j = 0; j < bn / box_cols; ++j)
+          tma_store_3d(&p.tmap_c, ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), n0 + j * box_cols,
+                       m0 + r0, b);
+        tma_store_commit_and_wait_read();
+      }
     }
+    if (trace && t == 0) trace[7] = stamp();
   }
-  if (trace && t == 0) trace[7] = globaltimer();
 
   // ---------------- teardown
   tc_fence_before();
   __syncthreads();
-  if (warp == 5) {
+  if (warp == kEpiWarps + 1) {
     tc_fence_after();
     tmem_dealloc(tmem_base, p.tmem_cols);
   }

@@ -10,7 +10,9 @@ namespace pask {
 
 constexpr int kBM = 128;       // UMMA M (cta_group::1): one TMEM lane per tile row
 constexpr int kBK = 64;        // 64 bf16 = 128 B = one SWIZZLE_128B row
-constexpr int kGemmThreads = 192;  // warps 0-3 gather/epilogue, 4 TMA, 5 TMEM+MMA
+constexpr int kEpiWarps = 8;       // warps 0-7: bias, gather (A_GATHER), epilogue
+constexpr int kEpiThreads = 32 * kEpiWarps;
+constexpr int kGemmThreads = kEpiThreads + 64;  // + warp 8 TMA producer, warp 9 TMEM + MMA
 
 // A-operand source of the contraction kernel.
 enum AMode : int32_t {
@@ -29,9 +31,10 @@ struct alignas(64) GemmParams {
   void* out;           // bf16 output (row i of tile at out + off_c + b*stride_c + i*ldc)
   const void* res;     // bf16 residual, same indexing as out (nullable)
   const float* bias;   // fp32 [N] (nullable)
-  float* ws_partial;   // split-K fp32 partial tiles
-  uint32_t* ws_counter;  // unused (split-K reduces on chip); kept for layout stability
-  unsigned long long* trace;  // debug: per-CTA %globaltimer phase stamps (null in production)
+  int32_t trace_clock;  // debug: 1 = trace stamps are SM clock64 cycles instead of %globaltimer ns
+  int32_t reserved0;
+  int64_t reserved1;
+  unsigned long long* trace;  // debug: per-CTA phase stamps (null in production)
   int64_t ldc, off_c, stride_c;
   int32_t M, N, K, batch;
   int32_t num_kb;        // ceil(K / 64)

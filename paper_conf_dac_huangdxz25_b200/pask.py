@@ -73,7 +73,8 @@ class Stats(C.Structure):
                 ("encode_ns", C.c_uint64), ("gpu_span_ns", C.c_uint64), ("gpu_busy_ns", C.c_uint64),
                 ("cold_wall_ns", C.c_uint64), ("infer_count", C.c_uint64), ("launches", C.c_uint64),
                 ("load_done_ns", C.c_uint64), ("infer_entry_ns", C.c_uint64),
-                ("first_launch_ns", C.c_uint64), ("last_launch_ns", C.c_uint64)]
+                ("first_launch_ns", C.c_uint64), ("last_launch_ns", C.c_uint64),
+                ("encode_begin_ns", C.c_uint64), ("encode_end_ns", C.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -82,7 +83,7 @@ class Stats(C.Structure):
 EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "pask_load_model",
            "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
            "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name",
-           "pask_kernel_timeline", "pask_node_times"]
+           "pask_kernel_timeline", "pask_node_times", "pask_promote"]
 TEST_EXPORTS = ["pask_test_fake_driver", "pask_test_fake_log"]   # include/pask_testing.h
 
 _lib = None
@@ -114,6 +115,7 @@ def lib():
         "pask_kernel_timeline": (C.c_int, [P, C.c_int32, C.POINTER(C.c_uint64),
                                            C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
         "pask_node_times": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int32]),
+        "pask_promote": (C.c_int, [P, C.c_int32, C.POINTER(C.c_int32)]),
         "pask_last_error": (C.c_char_p, []),
         "pask_test_fake_driver": (C.c_int, [C.c_int32, C.c_int32, C.c_int32]),
         "pask_test_fake_log": (C.c_int32, [C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.c_int32]),
@@ -233,6 +235,12 @@ class Context:
         a, b, c = C.c_uint64(), C.c_uint64(), C.c_uint64()
         _check(lib().pask_kernel_timeline(self.h, k, C.byref(a), C.byref(b), C.byref(c)))
         return a.value, b.value, c.value
+
+    def promote(self, target_catalog=-1):
+        """Idle-interval loading of skipped / specialised solutions."""
+        n = C.c_int32()
+        _check(lib().pask_promote(self.h, target_catalog, C.byref(n)))
+        return n.value
 
     def node_times(self):
         """Per-node GPU ns of the last instrumented inference (cfg.instrument = 1)."""

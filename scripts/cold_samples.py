@@ -32,7 +32,9 @@ SCHEMES = {
     # tuned library (per-problem specialised conv solutions)
     "baseline_tuned": dict(catalog=1, proactive=0, reuse=0),  # the paper's Baseline
     "pask_tuned": dict(catalog=1),                    # PASK over the tuned library
+    "pask_encfirst": dict(),                          # experiment: caller encodes, then uploads
 }
+SCHEME_ENV = {"pask_encfirst": {"PASK_ENCODE_FIRST": "1"}}
 
 
 def child(model, scheme, batch=1):
@@ -78,6 +80,8 @@ def child(model, scheme, batch=1):
                       "t_load_done_us": st["load_done_ns"] / 1e3, "t_infer_entry_us": st["infer_entry_ns"] / 1e3,
                       "t_first_launch_us": st["first_launch_ns"] / 1e3,
                       "t_last_launch_us": st["last_launch_ns"] / 1e3,
+                      "t_encode_begin_us": st["encode_begin_ns"] / 1e3,
+                      "t_encode_end_us": st["encode_end_ns"] / 1e3,
                       "timeline": tl}))
     ctx.close()
 
@@ -99,7 +103,8 @@ def main():
         for _ in range(a.n):
             r = subprocess.run([sys.executable, __file__, "--model", a.model, "--child", scheme,
                                 "--batch", str(a.batch)],
-                               capture_output=True, text=True, timeout=300)
+                               capture_output=True, text=True, timeout=300,
+                               env={**os.environ, **SCHEME_ENV.get(scheme, {})})
             line = [l for l in r.stdout.splitlines() if l.startswith("{")]
             if not line:
                 print(r.stderr[-2000:], file=sys.stderr)
@@ -119,7 +124,8 @@ def main():
               f"  hot {med['hot_us']:7.1f}  ratio {med['cold_over_hot']:5.2f}  kernels {med['kernels_loaded']:.0f}"
               f"  load {med['load_us']:6.1f} exposed {med['load_exposed_us']:6.1f} issue {med['issue_us']:6.1f}"
               f" gpu {med['gpu_span_us']:6.1f} | t: loads {med['t_load_done_us']:6.1f} infer {med['t_infer_entry_us']:6.1f}"
-              f" first {med['t_first_launch_us']:6.1f} last {med['t_last_launch_us']:6.1f}", flush=True)
+              f" first {med['t_first_launch_us']:6.1f} last {med['t_last_launch_us']:6.1f}"
+              f" encode [{med['t_encode_begin_us']:6.1f}, {med['t_encode_end_us']:6.1f}]", flush=True)
     print(json.dumps({"model": a.model, "schemes": out}))
 
 

@@ -11,7 +11,11 @@ from paper_conf_dac_huangdxz25_b200 import pask as P  # noqa: E402
 from paper_conf_dac_huangdxz25_b200.model import DeviceModel  # noqa: E402
 from workloads import build_model  # noqa: E402
 
-name = sys.argv[1] if len(sys.argv) > 1 else "resnet50"
+args = [a for a in sys.argv[1:] if not a.startswith("--")]
+CLOCK = "--clock" in sys.argv  # per-CTA phase durations in SM cycles (clock64) instead of %globaltimer
+name = args[0] if args else "resnet50"
+if CLOCK:
+    os.environ["PASK_TRACE_CLOCK"] = "1"
 spec, x = build_model(name)
 dm = DeviceModel(spec)
 dm.set_input(x)
@@ -45,6 +49,18 @@ for i in range(n):
     rows.append((i, len(t), rel[:, 0].min(), rel[:, 7].max(), np.median(rel[:, 2] - rel[:, 0]),
                  np.median(rel[:, 3] - rel[:, 2]), np.median(rel[:, 5] - rel[:, 3]),
                  np.median(rel[:, 6] - rel[:, 5]), np.median(rel[:, 7] - rel[:, 6])))
+if CLOCK:
+    print(f"{'node':>4} {'ctas':>4} | median SM cycles: prologue pre-wait first-load mainloop epi-1st-chunk epi-rest store")
+    for i in range(n):
+        t = tr[i]
+        t = t[t[:, 0] > 0]
+        if not len(t):
+            continue
+        d = lambda a, b: int(np.median(t[:, b] - t[:, a]))
+        L = spec["layers"][i]
+        desc = L["op"] + (str(tuple(L["w"].shape)) + f" s{L['stride'][0]}" if L["op"] == "conv" else "")
+        print(f"{i:4d} {len(t):4d} | {d(0,1):6d} {d(0,2):6d} {d(2,3):6d} {d(3,5):6d} {d(5,4):6d} {d(4,6):6d} {d(6,7):6d}  {desc}")
+    sys.exit(0)
 prev_end = None
 print(f"{'node':>4} {'ctas':>4} {'start':>8} {'end':>8} {'dur':>6} {'gap':>6} | pre-wait first-load mainloop epilogue store (median us)")
 for r in rows:

@@ -125,3 +125,37 @@ def test_model_hot_repeat_bitwise(name):
     for a, b in zip(outs1, outs2):
         np.testing.assert_array_equal(a, b)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["resnet50", "mobilenet_v2"])
+def test_promote_idle_interval(name):
+    """Idle-interval loading: after the cold inference the skipped
+    s* solutions are loaded and the reused nodes rebound; the next (hot, graph
+    re-captured) inference stays within tolerance and every contraction layer is
+    bitwise unchanged (a reused solution computes the same tiles in the same
+    order, R6).  Promoting further to the tuned catalog loads the
+    per-problem specialisations, again bitwise equal."""
+    import torch
+    spec, x = build_model(name)
+    dm, ctx, plan = run_model(spec, x)
+    before = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
+    reused = sum(1 for b in plan if b[3] == 1)
+    assert ctx.promote() == reused > 0
+    assert all(ctx.kernel_is_loaded(b[1]) for b in plan)
+    stream = torch.cuda.current_stream().cuda_stream
+    ctx.infer(stream)
+    ctx.sync()
+    errs = teacher_forced_errors(dm, spec, x)
+    assert max(e for _, _, e in errs) <= TOL
+    after = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
+    for L in spec["layers"]:
+        if L["op"] in ("conv", "linear"):
+            np.testing.assert_array_equal(before[L["out"]], after[L["out"]])
+    n = ctx.promote(target_catalog=1)
+    o = OP.execution_plan(OP.problems_from_spec(spec), reuse=False, catalog="tuned")
+    assert n > 0 and all(ctx.kernel_is_loaded(k) for k in o["loaded"])
+    ctx.infer(stream)
+    ctx.sync()
+    for L in spec["layers"]:
+        np.testing.assert_array_equal(after[L["out"]], dm.read_raw(L["out"]))
+    ctx.close()

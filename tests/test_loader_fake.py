@@ -128,3 +128,27 @@ def test_state_errors():
         ctx.load_model(dm.graph)             # one model per context
     assert ei.value.code == P.ESTATE
     ctx.close()
+
+
+def test_promote_loads_skipped_solutions_in_order():
+    """Idle-interval loading: the solutions Algorithm 1 skipped are
+    uploaded after the cold inference and the reused nodes rebound to them."""
+    P.test_fake_driver(True, load_us=0)
+    spec, _ = build_model("resnet50")
+    dm = DeviceModel(spec, alloc=False)
+    ctx = P.Context(0, P.config())
+    plan = ctx.load_model(dm.graph)
+    ctx.infer(0)
+    n = ctx.promote()
+    assert n == sum(1 for b in plan if b[3] == 1) == 34            # every reused node
+    ctx.infer(0)
+    ctx.sync()
+    log = P.test_fake_log()
+    loads = [k for k, kind in log if kind == 0]
+    assert loads[5:] == [P.K_CONV_1X1, P.K_POOL_GAVG]             # skipped s*, first-use order
+    hot = [k for k, kind in log if kind == 1][len(plan):]
+    assert hot == [b[1] for b in plan]                             # every node on its s*
+    assert ctx.promote() == 0                                      # idempotent
+    n_tuned = ctx.promote(target_catalog=1)
+    assert n_tuned == 53                                           # every conv -> its specialisation
+    ctx.close()
