@@ -70,7 +70,8 @@ __device__ __forceinline__ uint32_t ro_addr(uint32_t ro, int lb, int row, int co
 __device__ __forceinline__ int box_log2(int bn) { return bn >= 64 ? 6 : (bn == 32 ? 5 : 4); }
 
 // v = act(acc + bias + res) -> bf16 (RNE) for 16 columns [cb, cb+16) of tile row
-// `row`: staged in smem for the TMA store (c_tma) or stored directly.
+// `row`: staged in smem for the TMA tensor store (c_tma) or, for unaligned
+// output rows, stored directly.
 __device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint32_t ro, int lb, int m0,
                                       int n0, int b, int row, int cb, float (&v)[16]) {
 #pragma unroll
@@ -273,7 +274,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       // weights of the first min(nk, stages) k-blocks before griddepcontrol.wait
       // (they overlap the previous layer's tail); ring slots start empty.  An
       // activation B operand (attention QK^T / PV) must wait like A.
-      const int pre = p.b_const ? min(nk, stages) : 0;
+      const int pre = p.b_const ? min(min(nk, stages), p.pre_b > 0 ? p.pre_b : stages) : 0;
       for (int i = 0; i < pre; ++i) {
         const uint32_t sb = smem_base + i * stage_bytes + kABytes;
         const int kb = kb_begin + i;

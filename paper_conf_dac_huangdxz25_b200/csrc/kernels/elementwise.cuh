@@ -74,23 +74,20 @@ __device__ __forceinline__ void pool_body(const PoolParams& p) {
     for (int i = 0; i < 8; ++i) acc[i] = p.mode == 0 ? -INFINITY : 0.f;
     float cnt = 0.f;
     const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
+    const bool is_max = p.mode == 0;
+#pragma unroll 1
     for (int tap = p.per_warp ? lane : 0; tap < taps; tap += p.per_warp ? 32 : 1) {
-      const int r = tap / p.S, s = tap - (tap / p.S) * p.S;
+      const int r = tap / p.S, s = tap - r * p.S;
       const int ih = ih0 + r, iw = iw0 + s;
       if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;
       float f[8];
       unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), f);
       cnt += 1.f;
-      if (p.mode == 0) {
 #pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] = fmaxf(acc[i], f[i]);
-      } else {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] += f[i];
-      }
+      for (int i = 0; i < 8; ++i) acc[i] = is_max ? fmaxf(acc[i], f[i]) : acc[i] + f[i];
     }
     if (p.per_warp) {
-#pragma unroll
+#pragma unroll 1
       for (int o = 16; o > 0; o >>= 1) {
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
@@ -101,9 +98,9 @@ __device__ __forceinline__ void pool_body(const PoolParams& p) {
       }
     }
     if (p.mode == 1) {
-      const float div = p.count_include_pad ? static_cast<float>(taps) : cnt;
+      const float inv = 1.f / (p.count_include_pad ? static_cast<float>(taps) : cnt);
 #pragma unroll
-      for (int i = 0; i < 8; ++i) acc[i] = acc[i] / div;
+      for (int i = 0; i < 8; ++i) acc[i] *= inv;
     }
     if (!p.per_warp || lane == 0) reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(acc);
   }
@@ -211,6 +208,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
   const bool vec = (p.cols & 7) == 0;
   float m = -INFINITY, s = 0.f;
   if (vec) {
+#pragma unroll 1
     for (int c = lane * 8; c < p.cols; c += 256) {
       float f[8];
       unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
@@ -223,6 +221,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
       m = lm;
     }
   } else {
+#pragma unroll 1
     for (int c = lane; c < p.cols; c += 32) {
       const float v = __bfloat162float(x[c]) * p.scale;
       const float lm = fmaxf(m, v);
@@ -234,6 +233,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
   s = (m == -INFINITY) ? 0.f : s * __expf(m - gm);
   const float inv = 1.f / warp_sum(s);
   if (vec) {
+#pragma unroll 1
     for (int c = lane * 8; c < p.cols; c += 256) {
       float f[8];
       unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
@@ -242,6 +242,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
       *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f);
     }
   } else {
+#pragma unroll 1
     for (int c = lane; c < p.cols; c += 32)
       y[c] = __float2bfloat16_rn(__expf(__bfloat162float(x[c]) * p.scale - gm) * inv);
   }

@@ -32,7 +32,7 @@ struct alignas(64) GemmParams {
   const void* res;     // bf16 residual, same indexing as out (nullable)
   const float* bias;   // fp32 [N] (nullable)
   int32_t trace_clock;  // debug: 1 = trace stamps are SM clock64 cycles instead of %globaltimer ns
-  int32_t reserved0;
+  int32_t pre_b;        // weight k-blocks fetched before griddepcontrol.wait (0 = the whole ring)
   int64_t reserved1;
   unsigned long long* trace;  // debug: per-CTA phase stamps (null in production)
   int64_t ldc, off_c, stride_c;
