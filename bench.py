@@ -185,7 +185,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="pask", choices=["pask", "reference"])
     ap.add_argument("--model", default="resnet50",
-                    choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"])
+                    choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base", "bert_base_fa"])
     ap.add_argument("--batch", type=int, default=1, help="images per inference (Table II sweep)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
@@ -200,6 +200,8 @@ def main():
                     "implicit-GEMM kernel",
         "mobilenet_v2": "MobileNetV2 batch 1 224x224 (depthwise + pointwise convs) cold start",
         "bert_base": "BERT-base seq 128 batch 1 (GEMM + softmax + layernorm) cold start",
+        "bert_base_fa": "BERT-base seq 128 batch 1 cold start, attention fused (QK^T -> softmax -> PV "
+                        "in one kernel; SURVEY.md 8(f) NEXT #4)",
     }[args.model]
 
     world = int(os.environ.get("WORLD_SIZE", "1"))

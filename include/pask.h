@@ -73,7 +73,9 @@ typedef enum {
   PASK_OP_GEMM = 2,     /* batched C = act(A op(B) + bias + res)                      */
   PASK_OP_POOL = 3,     /* max / avg, windowed or global                              */
   PASK_OP_SOFTMAX = 4,  /* row softmax of scale * x                                   */
-  PASK_OP_LAYERNORM = 5 /* row LayerNorm, biased variance                             */
+  PASK_OP_LAYERNORM = 5, /* row LayerNorm, biased variance                            */
+  PASK_OP_ATTENTION = 6  /* fused multi-head scaled dot-product attention (QK^T ->
+                            softmax -> PV in one kernel)      */
 } pask_op;
 
 /* Activations are fused epilogues of conv / GEMM (the activation primitive of
@@ -98,7 +100,8 @@ typedef enum {
   PASK_K_GEMM = 6,       /* batched GEMM, tcgen05/TMEM; cat (GEMM, bf16, ROWMAJOR)      */
   PASK_K_SOFTMAX = 7,    /* cat (SOFTMAX, bf16, ROWMAJOR)                               */
   PASK_K_LAYERNORM = 8,  /* cat (LAYERNORM, bf16, ROWMAJOR)                             */
-  PASK_NUM_KERNELS = 9   /* size of the generic catalog; ids >= 9 are the per-problem
+  PASK_K_ATTENTION = 9,  /* fused attention, tcgen05/TMEM; cat (ATTENTION, bf16, ROWMAJOR) */
+  PASK_NUM_KERNELS = 10  /* size of the generic catalog; ids >= 10 are the per-problem
                             specialised conv solutions of the tuned catalog (one per
                             (R, S, stride, pad, dilation, C) of configs C1-C3, category
                             (CONV, bf16, NHWC), applicable to exactly that problem
@@ -136,6 +139,12 @@ typedef struct {
  *            window (r, s), stride, pad; global_pool = 1 means window = (h, w).
  * SOFTMAX  : rows = n*h*w of in0, cols = c: y = softmax(scale * x) per row.
  * LAYERNORM: rows of in0: y = (x - mean) / sqrt(var + eps) * gamma + beta, var biased.
+ * ATTENTION: in0 = packed QKV rows [batch * m][3 * n * kk] (Q | K | V, head h at
+ *            columns h*kk of each third), out = [batch * m][n * kk]; m = sequence
+ *            length, n = heads, kk = head dim, scale = softmax scale.  For b, head h,
+ *            query i:  out[b*m + i][h*kk + d] =
+ *              sum_j softmax_j(scale * sum_e Q[b*m+i][h*kk+e] K[b*m+j][h*kk+e]) V[b*m+j][h*kk+d]
+ *            (no mask), the composition of the qk -> softmax -> pv layers.
  *
  * solution: the statically chosen kernel s*_i carried by the lowered model
  * (".mgx ... the determined optimal solutions for each layer"),

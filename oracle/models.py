@@ -50,6 +50,8 @@ def run_layer(layer, ins, res=None):
         return ops.attn_qk(ins[0], layer["heads"], layer["head_dim"])
     if op == "pv":
         return ops.attn_pv(ins[0], ins[1], layer["heads"], layer["head_dim"])
+    if op == "attention":
+        return ops.attention(ins[0], layer["heads"], layer["head_dim"], layer["scale"])
     raise ValueError(f"unknown op {op}")
 
 
@@ -80,4 +82,7 @@ def model_flops(spec):
         elif op in ("qk", "pv"):
             s = shapes[layer["inputs"][-1]][0]
             tot += 2 * layer["heads"] * s * s * layer["head_dim"]
+        elif op == "attention":  # QK^T and PV
+            s = shapes[layer["inputs"][0]][0]
+            tot += 4 * layer["heads"] * s * s * layer["head_dim"]
     return tot

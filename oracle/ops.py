@@ -249,6 +249,26 @@ def attn_pv(probs, qkv, heads, head_dim):
     return out
 
 
+def attention(qkv, heads, head_dim, scale):
+    """Multi-head scaled dot-product attention without mask, the definition
+    Attention(Q, K, V) = softmax(scale * Q K^T) V per head (Vaswani et al. 2017,
+    eq. 1; BERT self-attention), over packed rows qkv = [Q | K | V], head h at
+    columns h*head_dim of each third.  Written out directly (fp64), not through
+    attn_qk / softmax / attn_pv."""
+    qkv = _f64(qkv)
+    hid = heads * head_dim
+    out = np.empty((qkv.shape[0], hid))
+    for h in range(heads):
+        cols = slice(h * head_dim, (h + 1) * head_dim)
+        q = qkv[:, :hid][:, cols]
+        k = qkv[:, hid:2 * hid][:, cols]
+        v = qkv[:, 2 * hid:][:, cols]
+        z = scale * (q @ k.T)
+        e = np.exp(z - z.max(axis=1, keepdims=True))
+        out[:, cols] = (e / e.sum(axis=1, keepdims=True)) @ v
+    return out
+
+
 # ---------------------------------------------------------------------------
 # input layout (SURVEY.md §8(c) item 7; PAPER.md:73 footnote 2 layout kernels)
 # ---------------------------------------------------------------------------

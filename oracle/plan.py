@@ -24,12 +24,13 @@ from __future__ import annotations
 import math
 
 # op classes
-LAYOUT, CONV, DWCONV, POOL, GEMM, SOFTMAX, LAYERNORM = range(7)
+LAYOUT, CONV, DWCONV, POOL, GEMM, SOFTMAX, LAYERNORM, ATTENTION = range(8)
 
 # kernel catalog ids
-K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN = range(9)
+K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN, K_ATTN = range(10)
 KERNEL_NAMES = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw",
-                "pask_pool", "pask_pool_gavg", "pask_gemm", "pask_softmax", "pask_layernorm"]
+                "pask_pool", "pask_pool_gavg", "pask_gemm", "pask_softmax", "pask_layernorm",
+                "pask_attention"]
 
 # Tuned catalog: one specialised conv solution per distinct dense
 # conv problem (R, S, stride, pad, dilation, C) of configs C1-C3, ids 9 + i in
@@ -40,7 +41,7 @@ SPECS = sorted([
 ] + [(1, 1, 2, 0, 1, c) for c in (256, 512, 1024)]
   + [(3, 3, 1, 1, 1, c) for c in (8, 16, 32, 64, 128, 256, 512)]
   + [(3, 3, 2, 1, 1, c) for c in (8, 128, 256, 512)] + [(7, 7, 2, 3, 1, 8)])
-N_GENERIC = 9
+N_GENERIC = 10
 KERNEL_NAMES = KERNEL_NAMES + ["pask_conv_spec_r%ds%du%dp%dd%dc%d" % sp for sp in SPECS]
 
 # category key (op class, dtype, layout): dtype 0 = bf16 compute path, layouts
@@ -55,6 +56,7 @@ CATEGORY = {
     K_GEMM: (GEMM, 0, 2),
     K_SOFTMAX: (SOFTMAX, 0, 2),
     K_LN: (LAYERNORM, 0, 2),
+    K_ATTN: (ATTENTION, 0, 2),
 }
 CATEGORY.update({N_GENERIC + i: (CONV, 0, 1) for i in range(len(SPECS))})
 
@@ -108,6 +110,9 @@ def is_applicable(kid, p):
         return op == SOFTMAX and 1 <= p["cols"] <= 16384
     if kid == K_LN:
         return op == LAYERNORM and p["cols"] % 8 == 0 and 8 <= p["cols"] <= 8192
+    if kid == K_ATTN:
+        return (op == ATTENTION and p["gk"] == 64 and 1 <= p["gm"] <= 256
+                and p["gn"] >= 1 and p["batch"] >= 1)
     raise ValueError(kid)
 
 
@@ -136,6 +141,8 @@ def static_choice(p, catalog="generic"):
         return K_SOFTMAX
     if op == LAYERNORM:
         return K_LN
+    if op == ATTENTION:
+        return K_ATTN
     raise ValueError(op)
 
 
@@ -199,6 +206,10 @@ def problems_from_spec(spec):
             hd = layer["head_dim"]
             p.update(op=GEMM, gm=s_, gn=hd, gk=s_, batch=heads, lda=s_, ldb=three_h,
                      off_a=0, off_b=2 * (three_h // 3))
+        elif op == "attention":
+            s_, three_h = shapes[layer["inputs"][0]]
+            p.update(op=ATTENTION, gm=s_, gn=layer["heads"], gk=layer["head_dim"], batch=1,
+                     lda=three_h)
         elif op in ("softmax", "layernorm"):
             shp = shapes[layer["inputs"][0]]
             cols = shp[-1]

@@ -82,6 +82,19 @@ struct alignas(16) DwParams {
   int32_t act;
 };
 
+// Fused attention (PASK_K_ATTENTION): one CTA per (128-query tile, head, sequence).
+struct alignas(64) AttnParams {
+  CUtensorMap tmap_qkv;  // 3-D {3H, S, batch} bf16, box {64, 64, 1}, SWIZZLE_128B
+  void* out;             // bf16 [batch][S][H]
+  int32_t S, heads, batch, H;
+  int32_t s_pad;         // S rounded up to 64 (key blocks; TMA zero-fills the tail)
+  float scale_log2e;     // softmax scale * log2(e) (exp2 form)
+  uint32_t idesc_qk;     // M=128, N=s_pad, A/B K-major
+  uint32_t idesc_pv;     // M=128, N=64, A K-major, B MN-major
+  uint32_t tmem_cols;    // power of two >= s_pad + 64
+  uint32_t smem_bytes;
+};
+
 struct alignas(16) RowParams {
   const void* x;  // bf16 [rows][cols]
   void* y;        // bf16 [rows][cols]

@@ -12,7 +12,7 @@
 
 namespace pask {
 
-enum OpClass : int32_t { OC_LAYOUT = 0, OC_CONV, OC_DWCONV, OC_POOL, OC_GEMM, OC_SOFTMAX, OC_LAYERNORM };
+enum OpClass : int32_t { OC_LAYOUT = 0, OC_CONV, OC_DWCONV, OC_POOL, OC_GEMM, OC_SOFTMAX, OC_LAYERNORM, OC_ATTENTION };
 
 struct Problem {
   int32_t op = 0;

@@ -188,6 +188,13 @@ class DeviceModel:
                            out=self.index[out], m=s_, n=dh, kk=s_, batch=heads, trans_b=0,
                            lda=s_, ldb=three_h, ldc=hid, off_a=0, off_b=2 * hid, off_c=0,
                            stride_a=s_ * s_, stride_b=dh, stride_c=dh, act=0, solution=sol)
+            elif op == "attention":
+                heads, dh = L["heads"], L["head_dim"]
+                s_, three_h = self.dims[x][2], self.dims[x][3]
+                hid = three_h // 3
+                self._new(out, (s_, hid), torch.bfloat16, P.ROWMAJOR, (1, 1, s_, hid), "matrix")
+                self._node(op=P.OP_ATTENTION, in0=self.index[x], out=self.index[out], m=s_,
+                           n=heads, kk=dh, batch=1, scale=L["scale"], solution=sol)
             else:
                 raise ValueError(op)
         self.inputs = [self.index[n] for n, _, _ in spec["inputs"]]

@@ -78,7 +78,7 @@ CFGS = [dict(), dict(search=1), dict(reuse=0), dict(milestone=5), dict(milestone
         dict(catalog=1), dict(catalog=1, reuse=0), dict(catalog=1, search=1)]
 
 
-@pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"])
+@pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base", "bert_base_fa"])
 def test_planner_matches_oracle_on_models(name):
     spec, _ = build_model(name)
     dm = DeviceModel(spec, alloc=False)

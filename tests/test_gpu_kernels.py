@@ -135,6 +135,22 @@ def test_attention_batched_gemm():
     _check_spec(b.spec())
 
 
+@pytest.mark.parametrize("s,heads", [(128, 12), (128, 1), (64, 2), (100, 3), (200, 4), (256, 2), (16, 1),
+                                     (1, 1), (77, 5)])
+def test_fused_attention(s, heads):
+    """pask_attention (QK^T -> softmax -> PV in one tcgen05 kernel) vs the fp64
+    attention definition, including sequence tails that are not multiples of the
+    64-key block / 128-query tile."""
+    b = _Builder("fattn", 8)
+    dh = 64
+    x = b.input((s, heads * dh), "bf16")
+    qkv = b.linear(x, 3 * heads * dh, w_std=0.08, b_std=0.02)
+    ctx = b.attention(qkv, heads, dh, 1 / math.sqrt(dh))
+    b.outputs = [ctx]
+    dm, plan = _check_spec(b.spec())
+    assert plan[-1][2] == P.K_ATTENTION
+
+
 @pytest.mark.parametrize("kind", ["max3s2p1", "max2s2", "avg3s1p1", "avg_global", "max_global"])
 def test_pool(kind):
     b = _Builder("pool", 7)

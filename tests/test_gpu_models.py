@@ -12,7 +12,7 @@ from .gpu_harness import TOL, run_model, teacher_forced_errors
 
 pytestmark = pytest.mark.gpu
 
-MODELS = ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"]
+MODELS = ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base", "bert_base_fa"]
 
 
 @pytest.mark.parametrize("name", MODELS)

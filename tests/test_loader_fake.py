@@ -34,7 +34,7 @@ MODES = [
 ]
 
 
-@pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "bert_base"])
+@pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "bert_base", "bert_base_fa"])
 @pytest.mark.parametrize("mode", MODES, ids=[str(m) for m in MODES])
 def test_load_order_and_launch_safety(name, mode):
     spec, _ = build_model(name)

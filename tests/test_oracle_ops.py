@@ -268,3 +268,40 @@ def test_attention_pieces_vs_torch():
     # cross-check against torch's fused attention in float64
     sdpa = F.scaled_dot_product_attention(t[0][None], t[1][None], t[2][None])[0]
     np.testing.assert_allclose(ctx, sdpa.permute(1, 0, 2).reshape(s, -1).numpy(), rtol=1e-10)
+
+
+# ---------------------------------------------------------------- fused attention
+def test_attention_vs_torch_sdpa_fp64():
+    """ops.attention against torch's scaled_dot_product_attention (an independent
+    library routine) in float64, several heads, S not a multiple of 16."""
+    rng = np.random.default_rng(11)
+    s, heads, dh = 37, 3, 64
+    qkv = rng.normal(size=(s, 3 * heads * dh))
+    scale = 1.0 / 8.0
+    got = ops.attention(qkv, heads, dh, scale)
+    t = torch.from_numpy(qkv).view(s, 3, heads, dh).permute(1, 2, 0, 3)  # [3][h][s][d]
+    ref = torch.nn.functional.scaled_dot_product_attention(t[0], t[1], t[2], scale=scale)
+    ref = ref.permute(1, 0, 2).reshape(s, heads * dh).numpy()
+    np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_attention_closed_forms():
+    """Q = 0: every key gets weight 1/S, output row = mean of V; one-hot
+    dominant key: output = that key's V row; equals the qk -> softmax -> pv chain."""
+    rng = np.random.default_rng(12)
+    s, heads, dh = 20, 2, 64
+    qkv = rng.normal(size=(s, 3 * heads * dh))
+    hid = heads * dh
+    q0 = qkv.copy()
+    q0[:, :hid] = 0.0
+    out = ops.attention(q0, heads, dh, 0.125)
+    np.testing.assert_allclose(out, np.broadcast_to(q0[:, 2 * hid:].mean(axis=0), out.shape), atol=1e-12)
+    big = qkv.copy()
+    big[:, :hid] = 0.0
+    big[:, hid:2 * hid] = 0.0
+    big[:, 0] = 1.0                 # head 0 query component 0
+    big[5, hid] = 1e4               # key 5 of head 0 dominates
+    out = ops.attention(big, heads, dh, 1.0)
+    np.testing.assert_allclose(out[:, :dh], np.broadcast_to(big[5, 2 * hid:2 * hid + dh], (s, dh)), atol=1e-9)
+    chain = ops.attn_pv(ops.softmax(ops.attn_qk(qkv, heads, dh), 0.125), qkv, heads, dh)
+    np.testing.assert_allclose(ops.attention(qkv, heads, dh, 0.125), chain, rtol=1e-12, atol=1e-12)

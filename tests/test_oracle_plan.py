@@ -50,6 +50,8 @@ def test_full_model_counts_match_survey():
         "mobilenet_v2": (["pask_layout", "pask_conv_igemm", "pask_conv_dw", "pask_pool_gavg",
                           "pask_gemm", "pask_softmax"], 40, 34, 34),
         "bert_base": (["pask_layernorm", "pask_gemm", "pask_softmax"], 3, 0, 0),
+        # NEXT #4: qk -> softmax -> pv fused; the attention solution replaces softmax
+        "bert_base_fa": (["pask_layernorm", "pask_gemm", "pask_attention"], 3, 0, 0),
     }
     for name, (loaded, q, h, lk) in expect.items():
         spec, _ = build_model(name)

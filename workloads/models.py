@@ -174,6 +174,15 @@ class _Builder:
                                 out=y, heads=heads, head_dim=head_dim))
         return y
 
+    def attention(self, qkv, heads, head_dim, scale):
+        """Fused multi-head attention over the packed QKV rows (the qk -> softmax ->
+        pv composition as one layer; SURVEY.md §8(f) NEXT #4)."""
+        s, _ = self.shape(qkv)
+        y = self.tensor((s, heads * head_dim))
+        self.layers.append(dict(op="attention", name=f"attn{len(self.layers)}", inputs=[qkv],
+                                out=y, heads=heads, head_dim=head_dim, scale=float(scale)))
+        return y
+
     def spec(self):
         return dict(name=self.name, inputs=self.inputs, outputs=self.outputs,
                     tensors=self.tensors, layers=self.layers)
@@ -262,16 +271,19 @@ def mobilenet_v2(seed_weights=1, hw=224, batch=1):
 # C4 BERT-base encoder, seq 128, batch 1 (BASELINE.json configs[3])
 # ---------------------------------------------------------------------------
 def bert_base(seed_weights=1, seq=128, hidden=768, heads=12, ffn=3072, nlayers=12,
-              eps=1e-12):
-    b = _Builder("bert_base", seed_weights)
+              eps=1e-12, fused_attention=False):
+    b = _Builder("bert_base_fa" if fused_attention else "bert_base", seed_weights)
     dh = hidden // heads
     x = b.input((seq, hidden), "bf16")          # embedding sum (no gather)
     h = b.layernorm(x, eps)
     for _ in range(nlayers):
         qkv = b.linear(h, 3 * hidden, w_std=0.02, b_std=0.02)
-        sc = b.qk(qkv, heads, dh)
-        pr = b.softmax(sc, scale=1.0 / math.sqrt(dh))
-        ctx = b.pv(pr, qkv, heads, dh)
+        if fused_attention:
+            ctx = b.attention(qkv, heads, dh, 1.0 / math.sqrt(dh))
+        else:
+            sc = b.qk(qkv, heads, dh)
+            pr = b.softmax(sc, scale=1.0 / math.sqrt(dh))
+            ctx = b.pv(pr, qkv, heads, dh)
         ao = b.linear(ctx, hidden, res=h, w_std=0.02, b_std=0.02)
         h1 = b.layernorm(ao, eps)
         f1 = b.linear(h1, ffn, act="gelu", w_std=0.02, b_std=0.02)
@@ -287,6 +299,8 @@ MODELS = {
     "resnet50": resnet50,
     "mobilenet_v2": mobilenet_v2,
     "bert_base": bert_base,
+    # C4 with the qk -> softmax -> pv chain fused into one attention layer (NEXT #4)
+    "bert_base_fa": lambda **kw: bert_base(fused_attention=True, **kw),
 }
 
 
