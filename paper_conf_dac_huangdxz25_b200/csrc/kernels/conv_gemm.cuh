@@ -188,6 +188,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int a_mode = Geo::amode(p);
   const bool gather = kAllowGather && (a_mode == A_GATHER);
   const bool im2col = kAllowGather && (a_mode == A_IM2COL);
+  const bool im2col8 = kAllowGather && (a_mode == A_IM2COL8);
   const int gR = Geo::R(p), gS = Geo::S(p), gSH = Geo::SH(p), gSW = Geo::SW(p);
   const int gPH = Geo::PH(p), gPW = Geo::PW(p), gDH = Geo::DH(p), gDW = Geo::DW(p), gC = Geo::C(p);
   (void)gR;
@@ -258,7 +259,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
       int iw = 0, ih = 0, in = 0, cc = 0, tr = 0, ts = 0;
       const int cpt = gC >> 6;  // 64-channel chunks per filter tap
-      if (kAllowGather && im2col) {
+      if (kAllowGather && (im2col || im2col8)) {
         const int pq = p.P * p.Q;
         in = m0 / pq;
         const int rem = m0 - in * pq;
@@ -266,10 +267,20 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const int qq = rem - pp * p.Q;
         iw = qq * gSW - gPW;
         ih = pp * gSH - gPH;
-        const int tap = kb_begin / cpt;
-        cc = kb_begin - tap * cpt;
-        tr = tap / gS;
-        ts = tap - tr * gS;
+        if (im2col) {
+          const int tap = kb_begin / cpt;
+          cc = kb_begin - tap * cpt;
+          tr = tap / gS;
+          ts = tap - tr * gS;
+        }
+      }
+      // im2col8: (tap, channel) of the next 8-channel chunk in K order, k = tap * C + c
+      int k8 = kb_begin * kBK, c8 = 0, r8 = 0, s8 = 0;
+      if (kAllowGather && im2col8) {
+        const int tap = k8 / gC;
+        c8 = k8 - tap * gC;
+        r8 = tap / gS;
+        s8 = tap - r8 * gS;
       }
       // weights of the first min(nk, stages) k-blocks before griddepcontrol.wait
       // (they overlap the previous layer's tail); ring slots start empty.  An
@@ -315,6 +326,24 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
               ++tr;
             }
           }
+        } else if (kAllowGather && im2col8) {
+          // eight 128-pixel x 8-channel boxes, box q at sa + q * 2 KB (no swizzle);
+          // chunks past K load tap 0 (finite data; B is zero-filled there)
+#pragma unroll 1
+          for (int q = 0; q < 8; ++q) {
+            const bool kv = k8 < p.K;
+            tma_load_im2col_4d(sa + q * 2048, &p.tmap_a, full0 + 8 * s, kv ? c8 : 0, iw, ih, in,
+                               static_cast<uint16_t>(kv ? s8 * gDW : 0), static_cast<uint16_t>(kv ? r8 * gDH : 0));
+            k8 += 8;
+            c8 += 8;
+            if (c8 == gC) {
+              c8 = 0;
+              if (++s8 == gS) {
+                s8 = 0;
+                ++r8;
+              }
+            }
+          }
         } else if (!gather) {
           tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
         }
@@ -347,8 +376,11 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const uint32_t sb = sa + kABytes;
 #pragma unroll
         for (int k = 0; k < kBK / 16; ++k) {
-          // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row
-          const uint64_t adesc = umma_desc_sw128(sa + k * 32, 16, 1024);
+          // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row;
+          // im2col8: no-swizzle core matrices, 8-channel boxes 2 KB apart along K,
+          // 8-row groups 128 B apart along M
+          const uint64_t adesc = im2col8 ? umma_desc_noswz(sa + k * 4096, 2048, 128)
+                                         : umma_desc_sw128(sa + k * 32, 16, 1024);
           const uint64_t bdesc = (p.b_major == 0)
                                      ? umma_desc_sw128(sb + k * 32, 16, 1024)
                                      // MN-major: +16 K rows of 128 B; 64-wide N chunks 8 KB apart

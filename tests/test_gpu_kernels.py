@@ -49,11 +49,13 @@ CONV_CASES = [
     (8, 48, 23, 7, 2, 3, 1, "none", False),        # bn 48, 7x7 s2 p3 (stem-like)
     (64, 64, 14, 3, 1, 2, 2, "relu", False),       # dilation 2
     (64, 256, 56, 1, 1, 0, 1, "relu", True),       # 1x1 TMA A path, residual TMA
-    (256, 128, 28, 1, 2, 0, 1, "none", False),     # 1x1 stride 2 -> gather path
+    (256, 128, 28, 1, 2, 0, 1, "none", False),     # 1x1 stride 2 -> TMA im2col path
     (512, 512, 7, 3, 1, 1, 1, "relu", True),       # M = 49, cluster split-K 8
     (1024, 256, 14, 1, 1, 0, 1, "relu", False),    # split-K 2..8 on a 1x1
     (128, 1000, 9, 3, 1, 1, 1, "gelu", True),      # N tail 1000 % 64, GELU epilogue
     (40, 24, 19, 5, 1, 2, 1, "tanh", False),       # C % 64 != 0 taps, tanh epilogue
+    (24, 64, 15, 3, 2, 1, 2, "relu", True),        # narrow-C TMA im2col, dilation + stride, residual
+    (96, 64, 10, 3, 1, 1, 1, "relu6", False),      # C = 1.5 x 64: eight 8-channel boxes per k-block
 ]
 
 
@@ -61,6 +63,22 @@ CONV_CASES = [
 def test_conv_cases(case):
     c, k, hw, r, s, p, d, act, res = case
     _check_spec(conv_spec(c, k, hw, r, s, p, d, act, res))
+
+
+@pytest.mark.parametrize("case", [CONV_CASES[i] for i in (0, 2, 3, 9, 10)], ids=str)
+def test_conv_gather_fallback(case, monkeypatch):
+    """The cp.async implicit-im2col gather, forced for every non-plain conv with
+    PASK_NO_IM2COL (the 64-channel TMA im2col cases then take it too)."""
+    monkeypatch.setenv("PASK_NO_IM2COL", "1")
+    _check_spec(conv_spec(*case))
+
+
+@pytest.mark.parametrize("case", [CONV_CASES[i] for i in (0, 1, 2, 9, 10, 11)], ids=str)
+def test_conv_narrow_tma_im2col(case, monkeypatch):
+    """A_IM2COL8 (eight 8-channel TMA im2col boxes per k-block, no-swizzle
+    core-matrix A operand), selected with PASK_IM2COL8 for narrow C."""
+    monkeypatch.setenv("PASK_IM2COL8", "1")
+    _check_spec(conv_spec(*case))
 
 
 @pytest.mark.parametrize("s,hw", [(1, 56), (2, 56), (1, 7), (2, 15)])
