@@ -101,7 +101,8 @@ typedef enum {
   PASK_K_SOFTMAX = 7,    /* cat (SOFTMAX, bf16, ROWMAJOR)                               */
   PASK_K_LAYERNORM = 8,  /* cat (LAYERNORM, bf16, ROWMAJOR)                             */
   PASK_K_ATTENTION = 9,  /* fused attention, tcgen05/TMEM; cat (ATTENTION, bf16, ROWMAJOR) */
-  PASK_NUM_KERNELS = 10  /* size of the generic catalog; ids >= 10 are the per-problem
+  PASK_K_CONV_IGEMM_PT = 10, /* implicit-GEMM conv as persistent tiles (large M); cat (CONV, bf16, NHWC) */
+  PASK_NUM_KERNELS = 11  /* size of the generic catalog; ids >= 11 are the per-problem
                             specialised conv solutions of the tuned catalog (one per
                             (R, S, stride, pad, dilation, C) of configs C1-C3, category
                             (CONV, bf16, NHWC), applicable to exactly that problem

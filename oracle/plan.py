@@ -27,10 +27,13 @@ import math
 LAYOUT, CONV, DWCONV, POOL, GEMM, SOFTMAX, LAYERNORM, ATTENTION = range(8)
 
 # kernel catalog ids
-K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN, K_ATTN = range(10)
+K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN, K_ATTN, K_IGEMM_PT = range(11)
 KERNEL_NAMES = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw",
                 "pask_pool", "pask_pool_gavg", "pask_gemm", "pask_softmax", "pask_layernorm",
-                "pask_attention"]
+                "pask_attention", "pask_conv_igemm_pt"]
+# s* of a dense conv with more output rows N*P*Q than 148 SMs x 128-row tiles is the
+# persistent-tile implicit-GEMM solution
+PERSISTENT_ROWS = 148 * 128
 
 # Tuned catalog: one specialised conv solution per distinct dense
 # conv problem (R, S, stride, pad, dilation, C) of configs C1-C3, ids 9 + i in
@@ -41,7 +44,7 @@ SPECS = sorted([
 ] + [(1, 1, 2, 0, 1, c) for c in (256, 512, 1024)]
   + [(3, 3, 1, 1, 1, c) for c in (8, 16, 32, 64, 128, 256, 512)]
   + [(3, 3, 2, 1, 1, c) for c in (8, 128, 256, 512)] + [(7, 7, 2, 3, 1, 8)])
-N_GENERIC = 10
+N_GENERIC = 11
 KERNEL_NAMES = KERNEL_NAMES + ["pask_conv_spec_r%ds%du%dp%dd%dc%d" % sp for sp in SPECS]
 
 # category key (op class, dtype, layout): dtype 0 = bf16 compute path, layouts
@@ -57,6 +60,7 @@ CATEGORY = {
     K_SOFTMAX: (SOFTMAX, 0, 2),
     K_LN: (LAYERNORM, 0, 2),
     K_ATTN: (ATTENTION, 0, 2),
+    K_IGEMM_PT: (CONV, 0, 1),
 }
 CATEGORY.update({N_GENERIC + i: (CONV, 0, 1) for i in range(len(SPECS))})
 
@@ -77,7 +81,7 @@ def is_applicable(kid, p):
     if kid == K_LAYOUT:
         return (op == LAYOUT and p["k"] % 8 == 0 and p["c"] <= p["k"]
                 and p["n"] * p["h"] * p["w"] * max(p["c"], p["k"]) < 2 ** 31)
-    if kid == K_IGEMM:
+    if kid in (K_IGEMM, K_IGEMM_PT):
         return (op == CONV and p["groups"] == 1 and p["c"] % 8 == 0 and p["k"] % 8 == 0
                 and 1 <= p["r"] <= 16 and 1 <= p["s"] <= 16
                 and 1 <= p["stride_h"] <= 8 and 1 <= p["stride_w"] <= 8
@@ -129,6 +133,8 @@ def static_choice(p, catalog="generic"):
     if op == DWCONV:
         return K_DW
     if op == CONV:
+        if p["n"] * p["p"] * p["q"] > PERSISTENT_ROWS:
+            return K_IGEMM_PT
         if (p["r"] == 1 and p["s"] == 1 and p["stride_h"] == 1 and p["stride_w"] == 1
                 and p["pad_h"] == 0 and p["pad_w"] == 0):
             return K_CONV1X1

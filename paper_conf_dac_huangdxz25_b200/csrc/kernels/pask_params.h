@@ -12,7 +12,8 @@ constexpr int kBM = 128;       // UMMA M (cta_group::1): one TMEM lane per tile 
 constexpr int kBK = 64;        // 64 bf16 = 128 B = one SWIZZLE_128B row
 constexpr int kEpiWarps = 8;       // warps 0-7: bias, gather (A_GATHER), epilogue
 constexpr int kEpiThreads = 32 * kEpiWarps;
-constexpr int kGemmThreads = kEpiThreads + 64;  // + warp 8 TMA producer, warp 9 TMEM + MMA
+constexpr int kGemmThreads = kEpiThreads + 64;    // + warp 8 TMA producer, warp 9 TMEM + MMA
+constexpr int kGemmThreadsPT = kEpiThreads + 96;  // persistent: + warp 10 store / residual agent
 
 // A-operand source of the contraction kernel.
 enum AMode : int32_t {
@@ -35,7 +36,8 @@ struct alignas(64) GemmParams {
   const float* bias;   // fp32 [N] (nullable)
   int32_t trace_clock;  // debug: 1 = trace stamps are SM clock64 cycles instead of %globaltimer ns
   int32_t pre_b;        // weight k-blocks fetched before griddepcontrol.wait (0 = the whole ring)
-  int64_t reserved1;
+  int32_t persistent;   // 1: grid of <= #SMs CTAs loops over the tiles, TMEM double-buffered
+  int32_t n_tiles_total;  // m_tiles * n_tiles * batch (persistent)
   unsigned long long* trace;  // debug: per-CTA phase stamps (null in production)
   int64_t ldc, off_c, stride_c;
   int32_t M, N, K, batch;

@@ -59,11 +59,17 @@ struct GemmTiling {
   int32_t M, N, K, batch;
   int32_t bn, m_tiles, n_tiles, num_kb, splits, rows_per, stages;
   uint32_t smem_bytes, tmem_cols;
+  int32_t persistent;  // 1: grid of min(tiles, #SMs) CTAs looping over tiles (splits == 1)
+  int32_t grid_x;      // persistent grid size
 };
 // Dynamic shared memory the contraction kernels may request (attribute set at load).
 constexpr uint32_t kMaxDynSmem = 220u * 1024u;
 // c_tma: output / residual go through smem staging + TMA (changes the smem size)
-GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma);
+GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma,
+                       int32_t persistent_kernel = 0);
+// s* rule: a dense conv with more output rows than 148 SMs x 128-row tiles takes
+// the persistent-tile solution (PASK_K_CONV_IGEMM_PT)
+constexpr int64_t kPersistentRows = 148 * 128;
 
 // Contraction view of a conv / GEMM problem (M, N, K, batch, b_major).
 bool contraction_shape(const Problem& p, const pask_node& node, int32_t* M, int32_t* N, int32_t* K,

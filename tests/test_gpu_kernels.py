@@ -259,3 +259,25 @@ def test_errors_fail_loudly():
     assert "not applicable" in str(ei.value)
     ctx.close()
     torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("c,k,hw,r,res", [(64, 128, 160, 3, True), (8, 64, 224, 7, False), (128, 256, 144, 1, True)])
+def test_persistent_tiles_bitwise(c, k, hw, r, res):
+    """pask_conv_igemm_pt (s* for N*P*Q > 148 x 128 rows): <= 148 CTAs loop over
+    the tiles with a double-buffered TMEM accumulator, staging tiles and a store
+    agent.  Each tile is computed with the same K order as the one-tile-per-CTA
+    kernel, so the outputs are bitwise equal; both within tolerance of the oracle."""
+    spec = conv_spec(c, k, hw, r, 1, r // 2, 1, "relu", res)
+    conv_li = len(spec["layers"]) - 1
+    xin = make_input(spec, 0)
+    dm, ctx, plan = run_model(spec, xin)
+    assert plan[conv_li][1] == P.K_CONV_IGEMM_PT and plan[conv_li][2] == P.K_CONV_IGEMM_PT
+    errs = teacher_forced_errors(dm, spec, xin)
+    assert max(e for _, _, e in errs) <= TOL, errs
+    out_pt = dm.read_raw(spec["outputs"][0])
+    ctx.close()
+    sols = {li: P.K_CONV_IGEMM for li, L in enumerate(spec["layers"]) if L["op"] == "conv"}
+    dm2, ctx2, plan2 = run_model(spec, xin, solutions=sols)
+    assert plan2[conv_li][2] == P.K_CONV_IGEMM
+    np.testing.assert_array_equal(dm2.read_raw(spec["outputs"][0]), out_pt)
+    ctx2.close()

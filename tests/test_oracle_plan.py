@@ -63,6 +63,12 @@ def test_full_model_counts_match_survey():
         spec, _ = build_model(name)
         pl = P.execution_plan(P.problems_from_spec(spec), search="naive")
         assert pl["lookups"] / pl["hits"] == pytest.approx(per_hit, abs=0.005)
+    # batch 128: dense convs with N*P*Q > 148*128 rows take the persistent-tile
+    # solution as s*; the smaller stage-3/4 convs reuse it (no conv_1x1 / igemm load)
+    spec, _ = build_model("resnet50", batch=128)
+    pl = P.execution_plan(P.problems_from_spec(spec))
+    assert [P.KERNEL_NAMES[k] for k in pl["loaded"]] == [
+        "pask_layout", "pask_conv_igemm_pt", "pask_pool", "pask_gemm", "pask_softmax"]
     # no reuse: ResNet-50 loads 7 distinct s* (adds conv_1x1 and gavg), MobileNetV2 7
     for name, n in (("resnet50", 7), ("mobilenet_v2", 7)):
         spec, _ = build_model(name)
