@@ -44,8 +44,7 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
 }
 
 // Activation over 16 values: ReLU / ReLU6 inline; GELU / tanh (transformer
-// GEMMs) through one out-of-line scalar routine (code size; passing the array
-// by address would put it in local memory for every path).
+// GEMMs) through one out-of-line routine to keep the code object small.
 __device__ __noinline__ float act_slow(float v, int act) { return apply_act(v, act); }
 __device__ __forceinline__ void act16(float (&v)[16], int act) {
   if (act == 1) {
@@ -85,14 +84,10 @@ __device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint3
     v[4 * q4 + 2] += bb.z;
     v[4 * q4 + 3] += bb.w;
   }
-  // residual: from the TMA-staged smem tile (c_tma) or from global (unaligned rows)
-  const uint32_t a0 = ro_addr(ro, lb, row, cb);
-  const uint32_t a1 = ro_addr(ro, lb, row, cb + 8);
-  const int m = m0 + row, n = n0 + cb;
-  const int nv = min(16, p.N - n);
-  const int64_t base = p.off_c + static_cast<int64_t>(b) * p.stride_c + static_cast<int64_t>(m) * p.ldc + n;
-  if (p.res) {
-    if (p.c_tma) {
+  if (p.c_tma) {
+    const uint32_t a0 = ro_addr(ro, lb, row, cb);
+    const uint32_t a1 = ro_addr(ro, lb, row, cb + 8);
+    if (p.res) {
       float f0[8], f1[8];
       unpack_bf16x8(lds_u4(a0), f0);
       unpack_bf16x8(lds_u4(a1), f1);
@@ -101,23 +96,26 @@ __device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint3
         v[i] += f0[i];
         v[8 + i] += f1[i];
       }
-    } else if (m < p.M) {
-      const __nv_bfloat16* res = reinterpret_cast<const __nv_bfloat16*>(p.res);
-#pragma unroll
-      for (int i = 0; i < 16; ++i)
-        if (i < nv) v[i] += __bfloat162float(res[base + i]);
     }
-  }
-  act16(v, p.act);
-  if (p.c_tma) {
+    act16(v, p.act);
     sts_u4(a0, pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
            pack_bf16x2(v[6], v[7]));
     sts_u4(a1, pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
            pack_bf16x2(v[14], v[15]));
     return;
   }
-  // unaligned output rows (e.g. N = 10): masked scalar stores
+  // unaligned output rows (e.g. N = 10): scalar stores, residual from global
+  const int m = m0 + row, n = n0 + cb;
   if (m >= p.M || n >= p.N) return;
+  const int nv = min(16, p.N - n);
+  const int64_t base = p.off_c + static_cast<int64_t>(b) * p.stride_c + static_cast<int64_t>(m) * p.ldc + n;
+  if (p.res) {
+    const __nv_bfloat16* res = reinterpret_cast<const __nv_bfloat16*>(p.res);
+#pragma unroll
+    for (int i = 0; i < 16; ++i)
+      if (i < nv) v[i] += __bfloat162float(res[base + i]);
+  }
+  act16(v, p.act);
   __nv_bfloat16* o = reinterpret_cast<__nv_bfloat16*>(p.out) + base;
 #pragma unroll
   for (int i = 0; i < 16; ++i)
@@ -157,8 +155,449 @@ struct FixGeo {
   }
 };
 
-template <bool kAllowGather, class Geo = DynGeo, bool kPersistent = false>
+
+template <bool kAllowGather, class Geo = DynGeo>
 __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const int t = threadIdx.x;
+  const int stages = p.stages;
+  const int bn = p.bn;
+  const int splits = p.splits;
+  constexpr uint32_t kABytes = kBM * kBK * 2;  // 16 KB
+  const uint32_t b_bytes = static_cast<uint32_t>(bn) * kBK * 2;
+  const uint32_t stage_bytes = kABytes + b_bytes;
+  // ---- smem carve-up (mirrors gemm_tiling() on the host)
+  const uint32_t ring_bytes = (stages * stage_bytes + 1023u) & ~1023u;
+  const uint32_t recv_pitch = (bn + 4) * 4;  // fp32 split-K receive row pitch (bank spread)
+  const uint32_t recv_bytes = splits > 1 ? ((128u * recv_pitch + 1023u) & ~1023u) : 0u;
+  const uint32_t reg0 = ring_bytes + recv_bytes;
+  const uint32_t ro_bytes = p.c_tma ? ((128u * bn * 2 + 1023u) & ~1023u) : 0u;
+  float* s_bias = reinterpret_cast<float*>(smem + reg0 + ro_bytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + reg0 + ro_bytes + 1024);
+  const uint32_t smem_base = smem_u32(smem);
+  const uint32_t full0 = smem_u32(bars);
+  const uint32_t empty0 = smem_u32(bars + stages);
+  const uint32_t accum_bar = smem_u32(bars + 2 * stages);
+  const uint32_t res_bar = smem_u32(bars + 2 * stages + 1);
+  const uint32_t recv_bar = smem_u32(bars + 2 * stages + 2);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * stages + 3);
+  const uint32_t ro = smem_base + reg0;
+  const uint32_t recv = smem_base + ring_bytes;  // slot s: rows [s*rows_per, (s+1)*rows_per)
+
+  const int a_mode = Geo::amode(p);
+  const bool gather = kAllowGather && (a_mode == A_GATHER);
+  const bool im2col = kAllowGather && (a_mode == A_IM2COL);
+  const int gR = Geo::R(p), gS = Geo::S(p), gSH = Geo::SH(p), gSW = Geo::SW(p);
+  const int gPH = Geo::PH(p), gPW = Geo::PW(p), gDH = Geo::DH(p), gDW = Geo::DW(p), gC = Geo::C(p);
+  (void)gR;
+  const int mt = blockIdx.x, nt = blockIdx.y;
+  const int b = blockIdx.z / splits;
+  const int split = blockIdx.z - b * splits;
+  const int kb_begin = static_cast<int>((static_cast<int64_t>(split) * p.num_kb) / splits);
+  const int kb_end = static_cast<int>((static_cast<int64_t>(split + 1) * p.num_kb) / splits);
+  const int nk = kb_end - kb_begin;  // >= 1 (host guarantees num_kb >= splits)
+  const int m0 = mt * kBM, n0 = nt * bn;
+  const int lb = box_log2(bn);
+  const int box_cols = 1 << lb;
+  const int rows_per = p.rows_per;
+  const int r0 = splits > 1 ? static_cast<int>(cluster_ctarank()) * rows_per : 0;
+  // rows of this tile inside the output, and of this rank's slice (split-K)
+  const int valid_rows = min(kBM, p.M - m0);
+  const int slice_rows = max(0, min(rows_per, valid_rows - r0));
+  const bool res_tma = p.c_tma && p.res != nullptr;
+  unsigned long long* trace =
+      p.trace ? p.trace + 8ull * (blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) : nullptr;
+  // debug phase stamps: [0] start [1] prologue done [2] producer past griddepcontrol.wait
+  // [3] first k-block landed [4] first accumulator chunk in registers (or split-K
+  // partials pushed) [5] accumulator ready [6] epilogue math done [7] tile stored
+  auto stamp = [&]() -> unsigned long long {
+    if (p.trace_clock) {
+      unsigned long long c;
+      asm volatile("mov.u64 %0, %%clock64;" : "=l"(c));
+      return c;
+    }
+    return globaltimer();
+  };
+  if (trace && t == 0) trace[0] = stamp();
+
+  // ---------------- prologue (overlaps the previous kernel under PDL)
+  if (t == 0) {
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(full0 + 8 * s, gather ? kEpiThreads + 1u : 1u);
+      mbar_init(empty0 + 8 * s, 1u);
+    }
+    mbar_init(accum_bar, 1u);
+    mbar_init(res_bar, 1u);
+    mbar_init(recv_bar, 1u);
+    if (splits > 1)  // the S-1 peers push the valid rows of this rank's slice, bn fp32 each
+      mbar_arrive_expect_tx(recv_bar, static_cast<uint32_t>((splits - 1) * slice_rows * bn * 4));
+    fence_barrier_init();
+  }
+  if (warp == kEpiWarps && lane == 0) {
+    if (!gather) tma_prefetch_desc(&p.tmap_a);
+    tma_prefetch_desc(&p.tmap_b);
+    if (p.c_tma) tma_prefetch_desc(&p.tmap_c);
+    if (res_tma) tma_prefetch_desc(&p.tmap_r);
+  }
+  if (warp == kEpiWarps + 1) tmem_alloc(smem_u32(tmem_slot), p.tmem_cols);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (splits > 1) cluster_sync_all();  // peers' receive barriers are initialised
+  const uint32_t tmem_base = *tmem_slot;
+  if (trace && t == 0) trace[1] = stamp();
+
+  pdl_launch_dependents();  // let the next layer's prologue start
+  // griddepcontrol.wait is per role: weights (B, bias) do not depend on the
+  // previous layer, so they are fetched before it; activations after it.
+
+  if (warp == kEpiWarps) {
+    // ================= TMA producer
+    if (lane == 0) {
+      // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
+      int iw = 0, ih = 0, in = 0, cc = 0, tr = 0, ts = 0;
+      const int cpt = gC >> 6;  // 64-channel chunks per filter tap
+      if (kAllowGather && im2col) {
+        const int pq = p.P * p.Q;
+        in = m0 / pq;
+        const int rem = m0 - in * pq;
+        const int pp = rem / p.Q;
+        const int qq = rem - pp * p.Q;
+        iw = qq * gSW - gPW;
+        ih = pp * gSH - gPH;
+        const int tap = kb_begin / cpt;
+        cc = kb_begin - tap * cpt;
+        tr = tap / gS;
+        ts = tap - tr * gS;
+      }
+      // weights of the first min(nk, stages) k-blocks before griddepcontrol.wait
+      // (they overlap the previous layer's tail); ring slots start empty.  An
+      // activation B operand (attention QK^T / PV) must wait like A.
+      const int pre = p.b_const ? min(min(nk, stages), p.pre_b > 0 ? p.pre_b : stages) : 0;
+      for (int i = 0; i < pre; ++i) {
+        const uint32_t sb = smem_base + i * stage_bytes + kABytes;
+        const int kb = kb_begin + i;
+        mbar_arrive_expect_tx(full0 + 8 * i, b_bytes + (gather ? 0u : kABytes));
+        if (p.b_major == 0) {
+          tma_load_3d(sb, &p.tmap_b, full0 + 8 * i, kb * kBK, n0, b);
+        } else {
+#pragma unroll 1
+          for (int j = 0; j < bn / 64; ++j)
+            tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * i, n0 + j * 64, kb * kBK, b);
+        }
+      }
+      pdl_wait();  // activations / residual of this layer are complete and visible
+      if (trace) trace[2] = stamp();
+      if (res_tma && slice_rows > 0) {  // residual rows [r0, r0 + rows_per), read by the epilogue
+        mbar_arrive_expect_tx(res_bar, static_cast<uint32_t>(rows_per * bn * 2));
+#pragma unroll 1
+        for (int j = 0; j < bn / box_cols; ++j)
+          tma_load_3d(ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), &p.tmap_r, res_bar,
+                      n0 + j * box_cols, m0 + r0, b);
+      }
+      int s = 0;
+      uint32_t ph = 0;
+      for (int i = 0; i < nk; ++i) {
+        const bool b_done = i < pre;
+        if (!b_done) mbar_wait(empty0 + 8 * s, ph ^ 1);
+        const uint32_t sa = smem_base + s * stage_bytes;
+        const uint32_t sb = sa + kABytes;
+        const int kb = kb_begin + i;
+        if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
+        if (kAllowGather && im2col) {
+          tma_load_im2col_4d(sa, &p.tmap_a, full0 + 8 * s, cc * 64, iw, ih, in,
+                             static_cast<uint16_t>(ts * gDW), static_cast<uint16_t>(tr * gDH));
+          if (++cc == cpt) {
+            cc = 0;
+            if (++ts == gS) {
+              ts = 0;
+              ++tr;
+            }
+          }
+        } else if (!gather) {
+          tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
+        }
+        if (!b_done) {
+          if (p.b_major == 0) {
+            tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
+          } else {
+#pragma unroll 1
+            for (int j = 0; j < bn / 64; ++j)
+              tma_load_3d(sb + j * 8192, &p.tmap_b, full0 + 8 * s, n0 + j * 64, kb * kBK, b);
+          }
+        }
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1;
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == kEpiWarps + 1) {
+    // ================= MMA issuer (one thread issues for the whole CTA)
+    if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0;
+      for (int i = 0; i < nk; ++i) {
+        mbar_wait(full0 + 8 * s, ph);
+        tc_fence_after();
+        if (trace && i == 0) trace[3] = stamp();
+        const uint32_t sa = smem_base + s * stage_bytes;
+        const uint32_t sb = sa + kABytes;
+#pragma unroll
+        for (int k = 0; k < kBK / 16; ++k) {
+          // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row
+          const uint64_t adesc = umma_desc_sw128(sa + k * 32, 16, 1024);
+          const uint64_t bdesc = (p.b_major == 0)
+                                     ? umma_desc_sw128(sb + k * 32, 16, 1024)
+                                     // MN-major: +16 K rows of 128 B; 64-wide N chunks 8 KB apart
+                                     : umma_desc_sw128(sb + k * 2048, 8192, 1024);
+          umma_f16(tmem_base, adesc, bdesc, p.idesc, (i | k) != 0 ? 1u : 0u);
+        }
+        umma_commit(empty0 + 8 * s);  // frees the smem slot when these MMAs complete
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1;
+        }
+      }
+      umma_commit(accum_bar);  // accumulator complete -> epilogue
+    }
+    __syncwarp();
+  } else {
+    // ================= warps 0-7: bias, (gather), epilogue
+    if (t < bn) s_bias[t] = (p.bias != nullptr && n0 + t < p.N) ? __ldg(p.bias + n0 + t) : 0.f;
+    pdl_wait();  // before reading this layer's activations (gather) or writing outputs
+    if (kAllowGather && gather) {
+      // implicit im2col: thread t owns 16 B chunk j = t % 8 of rows rg + kGR * ri
+      constexpr int kGR = kEpiThreads / 8;  // rows per pass
+      constexpr int kGI = kBM / kGR;        // passes per 128-row tile
+      const int j = t & 7;
+      const int rg = t >> 3;
+      const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x);
+      int ih0[kGI], iw0[kGI], nb[kGI];
+      bool rv[kGI];
+      {
+        // output pixel of row rg, then step kGR pixels per ri (no per-row divisions)
+        const int m = m0 + rg;
+        const int pq = p.P * p.Q;
+        int n = m / pq;
+        const int rem = m - n * pq;
+        int pp = rem / p.Q;
+        int qq = rem - pp * p.Q;
+#pragma unroll
+        for (int ri = 0; ri < kGI; ++ri) {
+          rv[ri] = (m + kGR * ri) < p.M;
+          ih0[ri] = pp * gSH - gPH;
+          iw0[ri] = qq * gSW - gPW;
+          nb[ri] = n * p.H;
+          qq += kGR;
+          while (qq >= p.Q) {
+            qq -= p.Q;
+            if (++pp == p.P) {
+              pp = 0;
+              ++n;
+            }
+          }
+        }
+      }
+      int kk = kb_begin * kBK + 8 * j;
+      int tap = kk / gC;
+      int c = kk - tap * gC;
+      int r = tap / gS;
+      int s = tap - r * gS;
+      const int lag = min(2, stages - 1);
+      int st = 0, st_lag = 0;  // ring slot being filled / being published
+      uint32_t ph = 0;
+      for (int i = 0; i < nk; ++i) {
+        mbar_wait(empty0 + 8 * st, ph ^ 1);
+        const uint32_t sa = smem_base + st * stage_bytes;
+        const bool kval = kk < p.K;
+        const int dih = r * gDH, diw = s * gDW;
+#pragma unroll
+        for (int ri = 0; ri < kGI; ++ri) {
+          const int row = rg + kGR * ri;
+          const uint32_t dst = sa + row * 128 + ((j ^ (row & 7)) << 4);
+          const int ih = ih0[ri] + dih;
+          const int iw = iw0[ri] + diw;
+          const bool ok = kval && rv[ri] && ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
+          const __nv_bfloat16* src =
+              ok ? x + ((static_cast<int64_t>(nb[ri] + ih) * p.W + iw) * gC + c) : x;
+          cp_async_16(dst, src, ok ? 16u : 0u);
+        }
+        cp_async_commit();
+        if (i >= lag) {
+          cp_async_wait_dyn(lag);
+          fence_proxy_async_smem();  // generic-proxy smem writes -> tcgen05 (async proxy)
+          mbar_arrive(full0 + 8 * st_lag);
+          if (++st_lag == stages) st_lag = 0;
+        }
+        if (++st == stages) {
+          st = 0;
+          ph ^= 1;
+        }
+        kk += kBK;
+        c += kBK;
+        while (c >= gC) {
+          c -= gC;
+          if (++s == gS) {
+            s = 0;
+            ++r;
+          }
+        }
+      }
+      cp_async_wait<0>();
+      fence_proxy_async_smem();
+      for (int i = max(0, nk - lag); i < nk; ++i) {
+        mbar_arrive(full0 + 8 * st_lag);
+        if (++st_lag == stages) st_lag = 0;
+      }
+    }
+    named_bar_sync(1, kEpiThreads);  // s_bias complete
+    mbar_wait(accum_bar, 0);
+    tc_fence_after();
+    if (trace && t == 0) trace[5] = stamp();
+  }
+
+  // ---------------- epilogue: warp w (0-7) reads TMEM lanes / tile rows
+  // 32*(w%4) .. +31 (the tcgen05.ld lane quarter of its warp) and the 16-column
+  // chunks c with c % 2 == w / 4.  Rows at or beyond M are never read or stored.
+  if (warp < kEpiWarps) {
+    const int quarter = warp & 3;
+    const int half = warp >> 2;
+    const int row = quarter * 32 + lane;
+    const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
+    const int cpr = bn >> 4;  // 16-column chunks per row
+    const uint32_t sbias = smem_u32(s_bias);
+    const bool warp_live = quarter * 32 < valid_rows;  // warp-uniform: tcgen05.ld is .sync.aligned
+    uint32_t r[16];
+    if (splits > 1) {
+      // push this split's fp32 partial rows to their owners' receive slot [my rank]
+      const uint32_t owner = static_cast<uint32_t>(row / rows_per);
+      const uint32_t me = cluster_ctarank();
+      const uint32_t slot_row = me * rows_per + (row - owner * rows_per);
+      const uint32_t local = recv + slot_row * recv_pitch;
+      const uint32_t remote = mapa_cluster(local, owner);
+      const uint32_t rbar = mapa_cluster(recv_bar, owner);
+      const bool live = row < valid_rows;
+      if (warp_live) {
+        int c = half;
+        if (c < cpr) {
+          tmem_ld16_issue(taddr + c * 16, r);
+          tmem_ld_wait(r);
+        }
+        for (; c < cpr; c += 2) {
+          uint32_t u[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) u[i] = r[i];
+          const bool more = c + 2 < cpr;
+          if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
+          if (live) {
+#pragma unroll
+            for (int q4 = 0; q4 < 4; ++q4) {
+              const uint32_t off = (c * 16 + 4 * q4) * 4;
+              const float x0 = __uint_as_float(u[4 * q4]), x1 = __uint_as_float(u[4 * q4 + 1]);
+              const float x2 = __uint_as_float(u[4 * q4 + 2]), x3 = __uint_as_float(u[4 * q4 + 3]);
+              if (owner == me)
+                sts_f4(local + off, x0, x1, x2, x3);
+              else
+                st_async_f4(remote + off, x0, x1, x2, x3, rbar);
+            }
+          }
+          if (more) tmem_ld_wait(r);
+        }
+      }
+      if (trace && t == 0) trace[4] = stamp();
+      named_bar_sync(1, kEpiThreads);  // own-slot rows visible to all epilogue threads
+      mbar_wait(recv_bar, 0);          // every peer's rows have landed
+      if (res_tma && slice_rows > 0) mbar_wait(res_bar, 0);
+    } else {
+      if (res_tma) mbar_wait(res_bar, 0);
+      if (warp_live && half < cpr) {
+        tmem_ld16_issue(taddr + half * 16, r);
+        tmem_ld_wait(r);
+        if (trace && t == 0) trace[4] = stamp();
+      }
+    }
+    // one epilogue loop (a single epi16 site keeps the code object small):
+    //   splits == 1: this warp's chunks c = half, half + 2, ..., TMEM reads software-
+    //                pipelined (chunk c + 2 in flight while c is processed);
+    //   splits  > 1: items (row, chunk) of this rank's slice, the S receive slots
+    //                summed in fixed rank order 0..S-1 (deterministic)
+    const int n_iter = splits == 1 ? (warp_live && half < cpr ? (cpr - half + 1) >> 1 : 0)
+                                   : max(0, (slice_rows * cpr - t + kEpiThreads - 1) / kEpiThreads);
+    for (int k = 0; k < n_iter; ++k) {
+      float v[16];
+      int erow, cb;
+      bool more = false;
+      if (splits == 1) {
+        const int c = half + 2 * k;
+        erow = row;
+        cb = c * 16;
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+        more = c + 2 < cpr;
+        if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
+      } else {
+        const int it = t + k * kEpiThreads;
+        const int lr = it / cpr;
+        erow = r0 + lr;
+        cb = (it - lr * cpr) << 4;
+        const uint32_t src = recv + lr * recv_pitch + cb * 4;
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = 0.f;
+        for (int sp = 0; sp < splits; ++sp) {
+          const uint32_t a = src + sp * rows_per * recv_pitch;
+#pragma unroll
+          for (int q4 = 0; q4 < 4; ++q4) {
+            const float4 f = lds_f4(a + 16 * q4);
+            v[4 * q4] += f.x;
+            v[4 * q4 + 1] += f.y;
+            v[4 * q4 + 2] += f.z;
+            v[4 * q4 + 3] += f.w;
+          }
+        }
+      }
+      if (erow < valid_rows) epi16(p, sbias, ro, lb, m0, n0, b, erow, cb, v);
+      if (more) tmem_ld_wait(r);
+    }
+    if (trace && t == 0) trace[6] = stamp();
+    if (p.c_tma) {
+      fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
+      named_bar_sync(1, kEpiThreads);
+      if (t == 0 && slice_rows > 0) {
+#pragma unroll 1
+        for (int j = 0; j < bn / box_cols; ++j)
+          tma_store_3d(&p.tmap_c, ro + j * (128 * box_cols * 2) + r0 * (box_cols * 2), n0 + j * box_cols,
+                       m0 + r0, b);
+        tma_store_commit_and_wait_read();
+      }
+    }
+    if (trace && t == 0) trace[7] = stamp();
+  }
+
+  // ---------------- teardown
+  tc_fence_before();
+  __syncthreads();
+  if (warp == kEpiWarps + 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem_base, p.tmem_cols);
+  }
+}
+
+
+// Persistent-tile variant (pask_conv_igemm_pt, DESIGN.md §6 K6-PT): when the grid
+// exceeds one wave, min(tiles, #SMs) CTAs loop over the tiles with double-buffered
+// TMEM accumulator / staging / bias and a store agent warp; otherwise one tile per
+// CTA.  Kept separate from conv_gemm_body so the one-tile solutions keep their
+// smaller, faster code (folding the loop into them cost 2-3% at batch 1).
+template <bool kAllowGather>
+__device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
+  using Geo = DynGeo;
+  constexpr bool kPersistent = true;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
@@ -200,7 +639,6 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int a_mode = Geo::amode(p);
   const bool gather = kAllowGather && (a_mode == A_GATHER);
   const bool im2col = kAllowGather && (a_mode == A_IM2COL);
-  const bool im2col8 = kAllowGather && (a_mode == A_IM2COL8);
   const int gR = Geo::R(p), gS = Geo::S(p), gSH = Geo::SH(p), gSW = Geo::SW(p);
   const int gPH = Geo::PH(p), gPW = Geo::PW(p), gDH = Geo::DH(p), gDW = Geo::DW(p), gC = Geo::C(p);
   (void)gR;
@@ -312,7 +750,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const int m0 = mt * kBM, n0 = nt * bn;
         // im2col: the tile's first output pixel and the (tap, channel chunk) of kb_begin
         int iw = 0, ih = 0, in = 0, cc = 0, tr = 0, ts = 0;
-        if (kAllowGather && (im2col || im2col8)) {
+        if (kAllowGather && im2col) {
           const int pq = p.P * p.Q;
           in = m0 / pq;
           const int rem = m0 - in * pq;
@@ -326,14 +764,6 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
             tr = tap / gS;
             ts = tap - tr * gS;
           }
-        }
-        // im2col8: (tap, channel) of the next 8-channel chunk in K order, k = tap * C + c
-        int k8 = kb_begin * kBK, c8 = 0, r8 = 0, s8 = 0;
-        if (kAllowGather && im2col8) {
-          const int tap = k8 / gC;
-          c8 = k8 - tap * gC;
-          r8 = tap / gS;
-          s8 = tap - r8 * gS;
         }
         int pre = 0;
         if (it == 0) {
@@ -372,24 +802,6 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
               if (++ts == gS) {
                 ts = 0;
                 ++tr;
-              }
-            }
-          } else if (kAllowGather && im2col8) {
-            // eight 128-pixel x 8-channel boxes, box q at sa + q * 2 KB (no swizzle);
-            // chunks past K load tap 0 (finite data; B is zero-filled there)
-#pragma unroll 1
-            for (int q = 0; q < 8; ++q) {
-              const bool kv = k8 < p.K;
-              tma_load_im2col_4d(sa + q * 2048, &p.tmap_a, full0 + 8 * s, kv ? c8 : 0, iw, ih, in,
-                                 static_cast<uint16_t>(kv ? s8 * gDW : 0), static_cast<uint16_t>(kv ? r8 * gDH : 0));
-              k8 += 8;
-              c8 += 8;
-              if (c8 == gC) {
-                c8 = 0;
-                if (++s8 == gS) {
-                  s8 = 0;
-                  ++r8;
-                }
               }
             }
           } else if (!gather) {
@@ -472,11 +884,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           const uint32_t sb = sa + kABytes;
 #pragma unroll
           for (int k = 0; k < kBK / 16; ++k) {
-            // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row;
-            // im2col8: no-swizzle core matrices, 8-channel boxes 2 KB apart along K,
-            // 8-row groups 128 B apart along M
-            const uint64_t adesc = im2col8 ? umma_desc_noswz(sa + k * 4096, 2048, 128)
-                                           : umma_desc_sw128(sa + k * 32, 16, 1024);
+            // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row
+            const uint64_t adesc = umma_desc_sw128(sa + k * 32, 16, 1024);
             const uint64_t bdesc = (p.b_major == 0)
                                        ? umma_desc_sw128(sb + k * 32, 16, 1024)
                                        // MN-major: +16 K rows of 128 B; 64-wide N chunks 8 KB apart

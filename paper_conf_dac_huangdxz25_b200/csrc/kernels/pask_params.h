@@ -20,8 +20,6 @@ enum AMode : int32_t {
   A_TMA = 0,     // A is a plain K-major matrix: TMA tiled load (GEMM, 1x1 s1 p0 conv)
   A_GATHER = 1,  // implicit im2col: cp.async gather with runtime pad/stride/dilation (any C % 8)
   A_IM2COL = 2,  // implicit im2col by TMA im2col mode (C % 64 == 0): one load per (tap, 64 ch)
-  A_IM2COL8 = 3, // TMA im2col for narrow C (C % 8 == 0): eight loads of (tap, 8 ch) x 128 px
-                 // per k-block into the no-swizzle K-major core-matrix layout
 };
 
 struct alignas(64) GemmParams {

@@ -269,18 +269,6 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr, uint32_t lbo
   return d;
 }
 
-// UMMA descriptor, K-major SWIZZLE_NONE (layout type 0): core matrices of
-// 8 rows x 16 B stored contiguously; lbo = byte stride between core matrices
-// along K, sbo = along M/N.
-__device__ __forceinline__ uint64_t umma_desc_noswz(uint32_t saddr, uint32_t lbo_bytes, uint32_t sbo_bytes) {
-  uint64_t d = 0;
-  d |= static_cast<uint64_t>((saddr >> 4) & 0x3FFF);
-  d |= static_cast<uint64_t>((lbo_bytes >> 4) & 0x3FFF) << 16;
-  d |= static_cast<uint64_t>((sbo_bytes >> 4) & 0x3FFF) << 32;
-  d |= 1ull << 46;
-  return d;
-}
-
 // ---------------------------------------------------------------- numerics
 // GELU (erf form) with the Abramowitz-Stegun 7.1.26 erf (|error| < 1.5e-7, far
 // below bf16 output resolution 2^-8) and tanh via tanh.approx.f32 (rel. error

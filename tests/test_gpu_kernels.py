@@ -54,8 +54,8 @@ CONV_CASES = [
     (1024, 256, 14, 1, 1, 0, 1, "relu", False),    # split-K 2..8 on a 1x1
     (128, 1000, 9, 3, 1, 1, 1, "gelu", True),      # N tail 1000 % 64, GELU epilogue
     (40, 24, 19, 5, 1, 2, 1, "tanh", False),       # C % 64 != 0 taps, tanh epilogue
-    (24, 64, 15, 3, 2, 1, 2, "relu", True),        # narrow-C TMA im2col, dilation + stride, residual
-    (96, 64, 10, 3, 1, 1, 1, "relu6", False),      # C = 1.5 x 64: eight 8-channel boxes per k-block
+    (24, 64, 15, 3, 2, 1, 2, "relu", True),        # narrow-C gather, dilation + stride, residual
+    (96, 64, 10, 3, 1, 1, 1, "relu6", False),      # C = 1.5 x 64 chunks: gather
 ]
 
 
@@ -70,14 +70,6 @@ def test_conv_gather_fallback(case, monkeypatch):
     """The cp.async implicit-im2col gather, forced for every non-plain conv with
     PASK_NO_IM2COL (the 64-channel TMA im2col cases then take it too)."""
     monkeypatch.setenv("PASK_NO_IM2COL", "1")
-    _check_spec(conv_spec(*case))
-
-
-@pytest.mark.parametrize("case", [CONV_CASES[i] for i in (0, 1, 2, 9, 10, 11)], ids=str)
-def test_conv_narrow_tma_im2col(case, monkeypatch):
-    """A_IM2COL8 (eight 8-channel TMA im2col boxes per k-block, no-swizzle
-    core-matrix A operand), selected with PASK_IM2COL8 for narrow C."""
-    monkeypatch.setenv("PASK_IM2COL8", "1")
     _check_spec(conv_spec(*case))
 
 
