@@ -191,8 +191,9 @@ def main():
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
                     help="1: hot inferences replay a CUDA graph captured on the 2nd call")
-    ap.add_argument("--packaging", type=int, default=0, choices=[0, 1],
-                    help="0: one code object per kernel (default); 1: whole catalog in one")
+    ap.add_argument("--packaging", type=int, default=0, choices=[0, 1, 2],
+                    help="0: one code object per kernel (default); 1: whole catalog in one; "
+                         "2: operator families (DESIGN.md D8)")
     args = ap.parse_args()
     args.workload_name = {
         "tiny_cnn": "tiny CNN 3xconv3x3(16/32/64)+maxpool+FC, 32x32x3, batch 1, bf16",
@@ -398,7 +399,8 @@ def main():
         "config": {"workload": args.workload_name, "model": args.model,
                    "global_batch": world * args.batch, "per_gpu_batch": args.batch,
                    "parallelism": f"replicas{world}",
-                   "packaging": ["one code object per kernel", "single code object"][args.packaging],
+                   "packaging": ["one code object per kernel", "single code object",
+                                 "operator families (memory-bound + contraction)"][args.packaging],
                    "hot_issue": "CUDA graph replay (captured on the 2nd inference)" if args.graph
                                 else "direct cuLaunchKernelEx per layer",
                    "l2": "warm (no flush)" if args.no_flush else

@@ -195,7 +195,13 @@ typedef struct {
   int32_t instrument; /* 1 = per-node CUDA events for gpu_busy_ns (perturbs timing)           */
   int32_t packaging;  /* 0 = one code object per catalog kernel (default: a load costs ~0.9 us
                          per KB of image, so only the bound kernels' code is parsed);
-                         1 = the whole catalog as one code object                            */
+                         1 = the whole catalog as one code object;
+                         2 = operator families (D8): the memory-bound solutions
+                             (layout, dw, pool, gavg, softmax, LayerNorm) share one
+                             CUfunction `pask_mem`, and conv_1x1 / gemm run on the generic
+                             implicit-GEMM function -- one upload makes a whole family
+                             resident; the plan (Algorithm 1) is unchanged, kernels_loaded
+                             counts the uploaded functions                                   */
   int32_t interleave; /* 0 = load-first (default): the first inference launches once every
                          planned kernel is uploaded -- on this driver a code upload waits for
                          all running GPU work, so

@@ -19,6 +19,25 @@ __device__ __forceinline__ float warp_max(float v) {
   return v;
 }
 
+// Activation over 8 values: ReLU / ReLU6 inline, GELU / tanh out of line (rare
+// on the memory-bound path; keeps the code object small -- uploads cost ~1.1 us
+// per KB of SASS).  Same arithmetic as apply_act either way.
+__device__ __noinline__ void act8_slow(float (&v)[8], int act) {
+#pragma unroll
+  for (int i = 0; i < 8; ++i) v[i] = apply_act(v[i], act);
+}
+__device__ __forceinline__ void act8(float (&v)[8], int act) {
+  if (act == 1) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = fmaxf(v[i], 0.f);
+  } else if (act == 2) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = fminf(fmaxf(v[i], 0.f), 6.f);
+  } else if (act >= 3) {
+    act8_slow(v, act);
+  }
+}
+
 // ---------------------------------------------------------------- K10 layout
 // NCHW fp32 -> NHWC bf16 (RNE), channels c..c_out-1 zero.  One thread per
 // (pixel, 8-channel chunk): coalesced fp32 reads across pixels, one 16 B store.
@@ -188,8 +207,7 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
 #pragma unroll
       for (int i = 0; i < 8; ++i) acc[i] += rf[i];
     }
-#pragma unroll
-    for (int i = 0; i < 8; ++i) acc[i] = apply_act(acc[i], p.act);
+    act8(acc, p.act);
     reinterpret_cast<uint4*>(p.y)[idx] = pack_bf16x8(acc);
   }
 }
@@ -250,7 +268,10 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
 
 // ---------------------------------------------------------------- K11 LayerNorm
 // One warp per row (cols % 8 == 0): mean, then biased variance of (x - mean)
-// (two passes over the row, fp32), then the affine transform.
+// (two passes over the row, fp32), then the affine transform.  Rows of up to
+// 1024 columns (BERT: 768) stay in registers: one load round trip instead of
+// three.  Both paths accumulate in the same order (lane's chunks ascending).
+constexpr int kLnRegChunks = 4;  // 16 B chunks per lane kept in registers
 __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   pdl_wait();
   pdl_launch_dependents();
@@ -259,7 +280,46 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   if (row >= p.rows) return;
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
+  if (p.cols <= 256 * kLnRegChunks) {
+    float f[kLnRegChunks][8];
+#pragma unroll
+    for (int j = 0; j < kLnRegChunks; ++j) {
+      const int c = lane * 8 + 256 * j;
+      if (c < p.cols) unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f[j]);
+    }
+    float s = 0.f;
+#pragma unroll
+    for (int j = 0; j < kLnRegChunks; ++j)
+      if (lane * 8 + 256 * j < p.cols) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) s += f[j][i];
+      }
+    const float mean = warp_sum(s) / static_cast<float>(p.cols);
+    float v = 0.f;
+#pragma unroll
+    for (int j = 0; j < kLnRegChunks; ++j)
+      if (lane * 8 + 256 * j < p.cols) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float d = f[j][i] - mean;
+          v = fmaf(d, d, v);
+        }
+      }
+    const float rstd = rsqrtf(warp_sum(v) / static_cast<float>(p.cols) + p.eps);
+#pragma unroll
+    for (int j = 0; j < kLnRegChunks; ++j) {
+      const int c = lane * 8 + 256 * j;
+      if (c < p.cols) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+          f[j][i] = (f[j][i] - mean) * rstd * __ldg(p.gamma + c + i) + __ldg(p.beta + c + i);
+        *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f[j]);
+      }
+    }
+    return;
+  }
   float s = 0.f;
+#pragma unroll 1
   for (int c = lane * 8; c < p.cols; c += 256) {
     float f[8];
     unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
@@ -268,6 +328,7 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   }
   const float mean = warp_sum(s) / static_cast<float>(p.cols);
   float v = 0.f;
+#pragma unroll 1
   for (int c = lane * 8; c < p.cols; c += 256) {
     float f[8];
     unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);
@@ -278,6 +339,7 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
     }
   }
   const float rstd = rsqrtf(warp_sum(v) / static_cast<float>(p.cols) + p.eps);
+#pragma unroll 1
   for (int c = lane * 8; c < p.cols; c += 256) {
     float f[8];
     unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f);

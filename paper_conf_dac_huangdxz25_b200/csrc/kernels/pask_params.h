@@ -107,4 +107,19 @@ struct alignas(16) RowParams {
   float eps;    // layernorm
 };
 
+// Operator-family entry (pask_config.packaging = 2): the memory-bound solutions
+// (layout, depthwise conv, pooling, softmax, LayerNorm) share ONE CUfunction,
+// `pask_mem`, so one code upload makes all of them resident.  The solution's
+// own parameter block sits at offset 0; `kind` selects its body.
+enum MemKind : int32_t { MEM_LAYOUT = 0, MEM_DW, MEM_POOL, MEM_GAVG, MEM_SOFTMAX, MEM_LAYERNORM };
+struct alignas(16) MemParams {
+  union {
+    LayoutParams l;
+    PoolParams p;
+    DwParams d;
+    RowParams r;
+  };
+  int32_t kind;  // MemKind
+};
+
 }  // namespace pask

@@ -83,7 +83,7 @@ def test_tuned_catalog_specialised_kernels(name):
     ctx2.close()
 
 
-@pytest.mark.parametrize("packaging", [0, 1])
+@pytest.mark.parametrize("packaging", [0, 1, 2])
 @pytest.mark.parametrize("cfg", ["reactive", "pask_i", "pask_r", "no_pdl"])
 def test_schemes_same_outputs(cfg, packaging):
     """Every scheme of PAPER.md:174-186 (reactive loading, PaSK-I = no reuse,
@@ -106,9 +106,35 @@ def test_schemes_same_outputs(cfg, packaging):
                           search="naive" if kw.get("search") else "categorical")
     assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
     st = ctx.stats()
-    assert st["kernels_loaded"] == len(o["loaded"])
-    assert st["code_objects_loaded"] == (1 if packaging == 1 else len(o["loaded"]))
+    if packaging == 2:   # ResNet-50's solutions fall in two families
+        assert st["kernels_loaded"] == st["code_objects_loaded"] == 2
+    else:
+        assert st["kernels_loaded"] == len(o["loaded"])
+        assert st["code_objects_loaded"] == (1 if packaging == 1 else len(o["loaded"]))
     ctx.close()
+
+
+@pytest.mark.parametrize("name", MODELS)
+def test_family_packaging_bitwise(name):
+    """Packaging 2 (D8): the same plan as packaging 0, every solution
+    resident (cuFuncIsLoaded) after at most one upload per operator family, and
+    every layer's output bitwise equal to the per-kernel code objects' (the family
+    entries run the same bodies on the same parameters)."""
+    spec, x = build_model(name)
+    dm, ctx, plan = run_model(spec, x, cfg=P.config(packaging=2))
+    o = OP.execution_plan(OP.problems_from_spec(spec))
+    assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
+    st = ctx.stats()
+    fams = {("mem" if k in (P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM)
+             else "contract" if k in (P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM) else k) for k in o["loaded"]}
+    assert st["kernels_loaded"] == st["code_objects_loaded"] == len(fams)
+    assert {k for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k)} >= set(o["loaded"])
+    fam_out = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
+    ctx.close()
+    dm2, ctx2, _ = run_model(spec, x)
+    for L in spec["layers"]:
+        np.testing.assert_array_equal(fam_out[L["out"]], dm2.read_raw(L["out"]))
+    ctx2.close()
 
 
 @pytest.mark.parametrize("name", MODELS)

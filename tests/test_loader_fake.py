@@ -31,7 +31,32 @@ MODES = [
     dict(proactive=2), dict(proactive=1), dict(proactive=1, interleave=1), dict(proactive=0),
     dict(proactive=2, packaging=1), dict(proactive=2, reuse=0), dict(proactive=1, search=1),
     dict(proactive=0, reuse=0, catalog=1), dict(proactive=2, catalog=1),
+    dict(proactive=2, packaging=2), dict(proactive=1, packaging=2), dict(proactive=0, packaging=2),
 ]
+
+# packaging 2 (D8): the CUfunction that serves a catalog solution, as
+# the fake driver logs it (the memory family entry `pask_mem` is id 63)
+FAM_MEM = 63
+MEM_SOLUTIONS = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM}
+CONTRACT_SOLUTIONS = {P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
+
+
+def function_of(k, packaging):
+    if packaging != 2:
+        return k
+    if k in MEM_SOLUTIONS:
+        return FAM_MEM
+    if k in CONTRACT_SOLUTIONS:
+        return P.K_CONV_IGEMM
+    return k
+
+
+def dedup(seq):
+    out = []
+    for x in seq:
+        if x not in out:
+            out.append(x)
+    return out
 
 
 @pytest.mark.parametrize("name", ["tiny_cnn", "resnet50", "bert_base", "bert_base_fa"])
@@ -53,11 +78,13 @@ def test_load_order_and_launch_safety(name, mode):
     exp = OP.execution_plan(OP.problems_from_spec(spec), reuse=bool(mode.get("reuse", 1)),
                             search="naive" if mode.get("search") else "categorical",
                             catalog="tuned" if mode.get("catalog") else "generic")
-    assert loads == exp["loaded"]                                   # once each, first-use order
+    pk = mode.get("packaging", 0)
+    want = dedup(function_of(k, pk) for k in exp["loaded"])
+    assert loads == want                                            # once each, first-use order
     assert all(kind == 1 for _, kind in launches)                   # never before its load
-    bound = [b[2] for b in plan]
+    bound = [function_of(b[2], pk) for b in plan]
     assert [k for k, _ in launches] == bound + bound                # node order, 2 inferences
-    assert st["kernels_loaded"] == len(exp["loaded"])
+    assert st["kernels_loaded"] == len(want)
     assert st["launches"] == 2 * len(bound)
     if mode.get("proactive", 2) == 2:
         assert st["load_exposed_ns"] == 0                           # all uploads inside load_model
