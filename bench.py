@@ -191,9 +191,9 @@ def main():
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
                     help="1: hot inferences replay a CUDA graph captured on the 2nd call")
-    ap.add_argument("--packaging", type=int, default=0, choices=[0, 1, 2],
-                    help="0: one code object per kernel (default); 1: whole catalog in one; "
-                         "2: operator families (DESIGN.md D8)")
+    ap.add_argument("--packaging", type=int, default=2, choices=[0, 1, 2],
+                    help="0: one code object per catalog kernel; 1: whole catalog in one; "
+                         "2 (default): operator families, DESIGN.md D8")
     args = ap.parse_args()
     args.workload_name = {
         "tiny_cnn": "tiny CNN 3xconv3x3(16/32/64)+maxpool+FC, 32x32x3, batch 1, bf16",
@@ -268,7 +268,9 @@ def main():
         if ld:
             timeline[P.kernel_name(k)] = {"load_us": round(ld / 1e3, 1), "ready_at_us": round(rd / 1e3, 1),
                                           "lib_us": round(lb / 1e3, 1)}
-    loaded = sorted(P.kernel_name(k) for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k))
+    solutions = sorted(P.kernel_name(k) for k in {b[2] for b in plan})  # Algorithm 1's bound set
+    loaded = sorted({P.function_name(k, args.packaging) for k in range(P.num_kernels())
+                     if ctx.kernel_is_loaded(k)})                       # CUfunctions resident
 
     # ---------------- warmup
     for _ in range(args.warmup):
@@ -412,6 +414,7 @@ def main():
         "hot_l2_warm_ms": round(warm_max, 4),
         "kernels_loaded": st["kernels_loaded"],
         "kernels_loaded_names": loaded,
+        "solutions_bound": solutions,
         "code_objects_loaded": st["code_objects_loaded"],
         "plan": {"queries": st["queries"], "hits": st["hits"], "lookups": st["lookups"],
                  "reused_nodes": sum(1 for b in plan if b[3] == 1)},

@@ -255,9 +255,11 @@ typedef struct {
 int pask_version(void);
 
 /* Create a context bound to the device's primary context (the one PyTorch
- * uses) and start the (idle) helper/loader thread.  cfg may be NULL for
- * defaults {reuse 1, search 0, milestone 0, proactive 2, pdl 1, instrument 0,
- * packaging 0, interleave 0}. */
+ * uses) and start the (idle) helper/loader thread.  Also touches the host pages
+ * of the embedded code objects this packaging may load (host residency of the
+ * library image, D8; nothing is uploaded to the GPU).  cfg may be
+ * NULL for defaults {reuse 1, search 0, milestone 0, proactive 2, pdl 1,
+ * instrument 0, packaging 0, interleave 0}. */
 int pask_create(pask_ctx **ctx, int device, const pask_config *cfg);
 
 /* Host-only planning (no GPU needed): validate g, extract problems p_i, apply
@@ -346,6 +348,12 @@ const char *pask_last_error(void);
 /* Catalog introspection (host only): total kernels (generic + specialised). */
 int32_t pask_num_kernels(void);
 const char *pask_kernel_name(int32_t kernel_id);
+/* Name of the CUfunction entry that serves catalog solution kernel_id under
+ * code-object packaging `packaging` (pask_config.packaging): its own entry for
+ * packaging 0 / 1; for packaging 2 the operator family's entry ("pask_mem" for
+ * layout / dw / pool / gavg / softmax / LayerNorm, "pask_conv_igemm" for
+ * igemm / conv_1x1 / gemm, D8).  "" for a bad id.  Host only. */
+const char *pask_kernel_function(int32_t kernel_id, int32_t packaging);
 
 #ifdef __cplusplus
 }

@@ -83,6 +83,7 @@ class Stats(C.Structure):
 EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "pask_load_model",
            "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
            "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name",
+           "pask_kernel_function",
            "pask_kernel_timeline", "pask_node_times", "pask_promote"]
 TEST_EXPORTS = ["pask_test_fake_driver", "pask_test_fake_log"]   # include/pask_testing.h
 
@@ -121,6 +122,7 @@ def lib():
         "pask_test_fake_log": (C.c_int32, [C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.c_int32]),
         "pask_num_kernels": (C.c_int32, []),
         "pask_kernel_name": (C.c_char_p, [C.c_int32]),
+        "pask_kernel_function": (C.c_char_p, [C.c_int32, C.c_int32]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -144,6 +146,11 @@ def _check(rc):
 
 def kernel_name(k):
     return lib().pask_kernel_name(k).decode()
+
+
+def function_name(k, packaging):
+    """CUfunction entry serving catalog solution k under a packaging (pask_kernel_function)."""
+    return lib().pask_kernel_function(k, packaging).decode()
 
 
 def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,

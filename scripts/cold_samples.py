@@ -26,8 +26,6 @@ SCHEMES = {
     "pask_interleave": dict(proactive=1, interleave=1),  # Fig. 5 interleaving
     "pask_single_image": dict(packaging=1),           # whole catalog as one code object
     "pask_families": dict(packaging=2),               # operator families (D8)
-    "pask_families_prewarm": dict(packaging=2),       # experiment: driver first-load cost paid in pask_create
-    "pask_prewarm": dict(),                           # experiment: same, per-kernel code objects
     "pask_i": dict(reuse=0),                          # PaSK-I: proactive, no reuse
     "pask_r": dict(search=1),                         # PaSK-R: naive (exhaustive-order) search
     "reactive": dict(proactive=0, reuse=0),           # Baseline analog: lazy load at first launch
@@ -37,8 +35,7 @@ SCHEMES = {
     "pask_tuned": dict(catalog=1),                    # PASK over the tuned library
     "pask_encfirst": dict(),                          # experiment: caller encodes, then uploads
 }
-SCHEME_ENV = {"pask_encfirst": {"PASK_ENCODE_FIRST": "1"}, "pask_families_prewarm": {"PASK_PREWARM": "1"},
-              "pask_prewarm": {"PASK_PREWARM": "1"}}
+SCHEME_ENV = {"pask_encfirst": {"PASK_ENCODE_FIRST": "1"}}
 
 
 def child(model, scheme, batch=1):

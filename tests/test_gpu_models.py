@@ -106,8 +106,8 @@ def test_schemes_same_outputs(cfg, packaging):
                           search="naive" if kw.get("search") else "categorical")
     assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
     st = ctx.stats()
-    if packaging == 2:   # ResNet-50's solutions fall in two families
-        assert st["kernels_loaded"] == st["code_objects_loaded"] == 2
+    if packaging == 2:   # ResNet-50's solutions fall in two families, one code object
+        assert st["kernels_loaded"] == 2 and st["code_objects_loaded"] == 1
     else:
         assert st["kernels_loaded"] == len(o["loaded"])
         assert st["code_objects_loaded"] == (1 if packaging == 1 else len(o["loaded"]))
@@ -127,7 +127,9 @@ def test_family_packaging_bitwise(name):
     st = ctx.stats()
     fams = {("mem" if k in (P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM)
              else "contract" if k in (P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM) else k) for k in o["loaded"]}
-    assert st["kernels_loaded"] == st["code_objects_loaded"] == len(fams)
+    assert st["kernels_loaded"] == len(fams)
+    # both families share one code object; other kernels keep their own
+    assert st["code_objects_loaded"] == len(fams - {"mem", "contract"}) + 1
     assert {k for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k)} >= set(o["loaded"])
     fam_out = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
     ctx.close()
