@@ -184,17 +184,40 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = 0.f;
     const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
-    for (int r = 0; r < p.R; ++r) {
-      const int ih = ih0 + r * p.dh;
-      if (ih < 0 || ih >= p.H) continue;
-      for (int s = 0; s < p.S; ++s) {
-        const int iw = iw0 + s * p.dw;
-        if (iw < 0 || iw >= p.W) continue;
+    if (p.R == 3 && p.S == 3 && p.dh == 1 && p.dw == 1) {
+      // 3x3 (MobileNetV2): all nine tap loads issued before the first FMA (one
+      // memory round trip instead of nine); same taps, same order as below
+      uint4 xv[9], wv[9];
+      bool ok[9];
+#pragma unroll
+      for (int t9 = 0; t9 < 9; ++t9) {
+        const int ih = ih0 + t9 / 3, iw = iw0 + t9 % 3;
+        ok[t9] = ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
+        xv[t9] = ok[t9] ? __ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch) : make_uint4(0, 0, 0, 0);
+        wv[t9] = __ldg(w + t9 * chunks + ch);
+      }
+#pragma unroll
+      for (int t9 = 0; t9 < 9; ++t9) {
+        if (!ok[t9]) continue;
         float xf[8], wf[8];
-        unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), xf);
-        unpack_bf16x8(__ldg(w + (r * p.S + s) * chunks + ch), wf);
+        unpack_bf16x8(xv[t9], xf);
+        unpack_bf16x8(wv[t9], wf);
 #pragma unroll
         for (int i = 0; i < 8; ++i) acc[i] = fmaf(xf[i], wf[i], acc[i]);
+      }
+    } else {
+      for (int r = 0; r < p.R; ++r) {
+        const int ih = ih0 + r * p.dh;
+        if (ih < 0 || ih >= p.H) continue;
+        for (int s = 0; s < p.S; ++s) {
+          const int iw = iw0 + s * p.dw;
+          if (iw < 0 || iw >= p.W) continue;
+          float xf[8], wf[8];
+          unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), xf);
+          unpack_bf16x8(__ldg(w + (r * p.S + s) * chunks + ch), wf);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) acc[i] = fmaf(xf[i], wf[i], acc[i]);
+        }
       }
     }
     if (p.bias) {
@@ -215,6 +238,7 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
 // ---------------------------------------------------------------- K11 softmax
 // One warp per row.  Pass 1: online max / sum of exp(scale*x - max) in fp32;
 // pass 2: write exp(scale*x - max) / sum as bf16.
+constexpr int kSmRegChunks = 4;  // 16 B chunks per lane kept in registers (rows <= 1024)
 __device__ __forceinline__ void softmax_body(const RowParams& p) {
   pdl_wait();
   pdl_launch_dependents();
@@ -225,6 +249,38 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
   const bool vec = (p.cols & 7) == 0;
   float m = -INFINITY, s = 0.f;
+  if (vec && p.cols <= 256 * kSmRegChunks) {
+    // short rows (BERT attention: 128, classifiers: 1000): the row stays in
+    // registers, one load round trip; same arithmetic order as the loop below
+    float f[kSmRegChunks][8];
+#pragma unroll
+    for (int j = 0; j < kSmRegChunks; ++j) {
+      const int c = lane * 8 + 256 * j;
+      if (c < p.cols) {
+        unpack_bf16x8(*reinterpret_cast<const uint4*>(x + c), f[j]);
+        float lm = m;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) lm = fmaxf(lm, f[j][i] * p.scale);
+        s *= __expf(m - lm);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) s += __expf(f[j][i] * p.scale - lm);
+        m = lm;
+      }
+    }
+    const float gm = warp_max(m);
+    s = (m == -INFINITY) ? 0.f : s * __expf(m - gm);
+    const float inv = 1.f / warp_sum(s);
+#pragma unroll
+    for (int j = 0; j < kSmRegChunks; ++j) {
+      const int c = lane * 8 + 256 * j;
+      if (c < p.cols) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) f[j][i] = __expf(f[j][i] * p.scale - gm) * inv;
+        *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f[j]);
+      }
+    }
+    return;
+  }
   if (vec) {
 #pragma unroll 1
     for (int c = lane * 8; c < p.cols; c += 256) {
@@ -270,7 +326,8 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
 // One warp per row (cols % 8 == 0): mean, then biased variance of (x - mean)
 // (two passes over the row, fp32), then the affine transform.  Rows of up to
 // 1024 columns (BERT: 768) stay in registers: one load round trip instead of
-// three.  Both paths accumulate in the same order (lane's chunks ascending).
+// three (gamma / beta 16 B aligned: vector loads).  Both paths accumulate in
+// the same order (lane's chunks ascending).
 constexpr int kLnRegChunks = 4;  // 16 B chunks per lane kept in registers
 __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   pdl_wait();
@@ -280,7 +337,8 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   if (row >= p.rows) return;
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
-  if (p.cols <= 256 * kLnRegChunks) {
+  const bool gb16 = ((reinterpret_cast<uintptr_t>(p.gamma) | reinterpret_cast<uintptr_t>(p.beta)) & 15) == 0;
+  if (p.cols <= 256 * kLnRegChunks && gb16) {
     float f[kLnRegChunks][8];
 #pragma unroll
     for (int j = 0; j < kLnRegChunks; ++j) {
@@ -310,9 +368,13 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
     for (int j = 0; j < kLnRegChunks; ++j) {
       const int c = lane * 8 + 256 * j;
       if (c < p.cols) {
+        const float4* g4 = reinterpret_cast<const float4*>(p.gamma + c);
+        const float4* b4 = reinterpret_cast<const float4*>(p.beta + c);
+        const float4 g0 = __ldg(g4), g1 = __ldg(g4 + 1), b0 = __ldg(b4), b1 = __ldg(b4 + 1);
+        const float g[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
+        const float be[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-        for (int i = 0; i < 8; ++i)
-          f[j][i] = (f[j][i] - mean) * rstd * __ldg(p.gamma + c + i) + __ldg(p.beta + c + i);
+        for (int i = 0; i < 8; ++i) f[j][i] = (f[j][i] - mean) * rstd * g[i] + be[i];
         *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f[j]);
       }
     }

@@ -73,7 +73,11 @@ def child(model, scheme, batch=1):
         ctx.infer(s)
     e1.record()
     torch.cuda.synchronize()
-    print(json.dumps({"cold_us": st["cold_wall_ns"] / 1e3, "cold_py_us": (t1 - t0) / 1e3, "hot_us": 1e3 * e0.elapsed_time(e1) / 50,
+    st2 = ctx.stats()
+    hot_issue = (st2["issue_ns"] - st["issue_ns"]) / 1e3 / max(1, st2["launches"] - st["launches"])
+    print(json.dumps({"hot_issue_us_per_launch": hot_issue,
+                      "cold_issue_us_per_launch": st["issue_ns"] / 1e3 / max(1, st["launches"]),
+                      "cold_us": st["cold_wall_ns"] / 1e3, "cold_py_us": (t1 - t0) / 1e3, "hot_us": 1e3 * e0.elapsed_time(e1) / 50,
                       "kernels_loaded": st["kernels_loaded"], "code_objects": st["code_objects_loaded"],
                       "load_us": st["load_ns"] / 1e3, "load_exposed_us": st["load_exposed_ns"] / 1e3,
                       "issue_us": st["issue_ns"] / 1e3, "gpu_span_us": st["gpu_span_ns"] / 1e3,
@@ -124,7 +128,8 @@ def main():
         print(f"{a.model:12s} {scheme:18s} cold med {med['cold_us']:8.1f} p90 {med['cold_p90_us']:8.1f} us"
               f"  hot {med['hot_us']:7.1f}  ratio {med['cold_over_hot']:5.2f}  kernels {med['kernels_loaded']:.0f}"
               f"  load {med['load_us']:6.1f} exposed {med['load_exposed_us']:6.1f} issue {med['issue_us']:6.1f}"
-              f" gpu {med['gpu_span_us']:6.1f} | t: loads {med['t_load_done_us']:6.1f} infer {med['t_infer_entry_us']:6.1f}"
+              f" gpu {med['gpu_span_us']:6.1f} issue/launch cold {med['cold_issue_us_per_launch']:4.2f}"
+              f" hot {med['hot_issue_us_per_launch']:4.2f} | t: loads {med['t_load_done_us']:6.1f} infer {med['t_infer_entry_us']:6.1f}"
               f" first {med['t_first_launch_us']:6.1f} last {med['t_last_launch_us']:6.1f}"
               f" encode [{med['t_encode_begin_us']:6.1f}, {med['t_encode_end_us']:6.1f}]", flush=True)
     print(json.dumps({"model": a.model, "schemes": out}))
