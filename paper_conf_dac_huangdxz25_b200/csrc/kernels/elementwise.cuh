@@ -94,16 +94,43 @@ __device__ __forceinline__ void pool_body(const PoolParams& p) {
     float cnt = 0.f;
     const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
     const bool is_max = p.mode == 0;
-#pragma unroll 1
-    for (int tap = p.per_warp ? lane : 0; tap < taps; tap += p.per_warp ? 32 : 1) {
-      const int r = tap / p.S, s = tap - r * p.S;
-      const int ih = ih0 + r, iw = iw0 + s;
-      if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;
-      float f[8];
-      unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), f);
-      cnt += 1.f;
+    if (!p.per_warp && taps <= 9) {
+      // small windows (ResNet-50's 3x3 max pool): every tap load issued before
+      // the first combine; same taps, same order as the loop below
+      uint4 xv[9];
+      bool ok[9];
+      int r = 0, s = 0;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) acc[i] = is_max ? fmaxf(acc[i], f[i]) : acc[i] + f[i];
+      for (int tap = 0; tap < 9; ++tap) {
+        const int ih = ih0 + r, iw = iw0 + s;
+        ok[tap] = tap < taps && ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
+        xv[tap] = ok[tap] ? __ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch) : make_uint4(0, 0, 0, 0);
+        if (++s == p.S) {
+          s = 0;
+          ++r;
+        }
+      }
+#pragma unroll
+      for (int tap = 0; tap < 9; ++tap) {
+        if (!ok[tap]) continue;
+        float f[8];
+        unpack_bf16x8(xv[tap], f);
+        cnt += 1.f;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = is_max ? fmaxf(acc[i], f[i]) : acc[i] + f[i];
+      }
+    } else {
+#pragma unroll 1
+      for (int tap = p.per_warp ? lane : 0; tap < taps; tap += p.per_warp ? 32 : 1) {
+        const int r = tap / p.S, s = tap - r * p.S;
+        const int ih = ih0 + r, iw = iw0 + s;
+        if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;
+        float f[8];
+        unpack_bf16x8(__ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch), f);
+        cnt += 1.f;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = is_max ? fmaxf(acc[i], f[i]) : acc[i] + f[i];
+      }
     }
     if (p.per_warp) {
 #pragma unroll 1
@@ -142,6 +169,8 @@ __device__ __forceinline__ void gavg_body(const PoolParams& p) {
   for (int i = 0; i < 8; ++i) acc[i] = 0.f;
   if (ch < chunks) {
     const uint4* x = reinterpret_cast<const uint4*>(p.x) + static_cast<int64_t>(n) * hw * chunks + ch;
+    // unrolled: four loads in flight per warp, the sum still in pixel order
+#pragma unroll 4
     for (int px = wq; px < hw; px += 4) {
       float f[8];
       unpack_bf16x8(__ldg(x + static_cast<int64_t>(px) * chunks), f);
