@@ -467,7 +467,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   // chunks c with c % 2 == w / 4.  Rows at or beyond M are never read or stored.
   if (warp < kEpiWarps) {
     const int quarter = warp & 3;
-    const int half = warp >> 2;
+    const int half = warp >> 2;  // warp group 0..kEpiGroups-1: chunks half, half + kEpiGroups, ...
     const int row = quarter * 32 + lane;
     const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
     const int cpr = bn >> 4;  // 16-column chunks per row
@@ -489,12 +489,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           tmem_ld16_issue(taddr + c * 16, r);
           tmem_ld_wait(r);
         }
-        for (; c < cpr; c += 2) {
+        for (; c < cpr; c += kEpiGroups) {
           uint32_t u[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i) u[i] = r[i];
-          const bool more = c + 2 < cpr;
-          if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
+          const bool more = c + kEpiGroups < cpr;
+          if (more) tmem_ld16_issue(taddr + (c + kEpiGroups) * 16, r);
           if (live) {
 #pragma unroll
             for (int q4 = 0; q4 < 4; ++q4) {
@@ -523,24 +523,24 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       }
     }
     // one epilogue loop (a single epi16 site keeps the code object small):
-    //   splits == 1: this warp's chunks c = half, half + 2, ..., TMEM reads software-
-    //                pipelined (chunk c + 2 in flight while c is processed);
+    //   splits == 1: this warp's chunks c = half, half + G, ... (G = kEpiGroups), TMEM
+    //                reads software-pipelined (chunk c + G in flight while c is processed);
     //   splits  > 1: items (row, chunk) of this rank's slice, the S receive slots
     //                summed in fixed rank order 0..S-1 (deterministic)
-    const int n_iter = splits == 1 ? (warp_live && half < cpr ? (cpr - half + 1) >> 1 : 0)
+    const int n_iter = splits == 1 ? (warp_live && half < cpr ? (cpr - half + kEpiGroups - 1) / kEpiGroups : 0)
                                    : max(0, (slice_rows * cpr - t + kEpiThreads - 1) / kEpiThreads);
     for (int k = 0; k < n_iter; ++k) {
       float v[16];
       int erow, cb;
       bool more = false;
       if (splits == 1) {
-        const int c = half + 2 * k;
+        const int c = half + kEpiGroups * k;
         erow = row;
         cb = c * 16;
 #pragma unroll
         for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
-        more = c + 2 < cpr;
-        if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
+        more = c + kEpiGroups < cpr;
+        if (more) tmem_ld16_issue(taddr + (c + kEpiGroups) * 16, r);
       } else {
         const int it = t + k * kEpiThreads;
         const int lr = it / cpr;
@@ -703,14 +703,14 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
   // ---------------- prologue (overlaps the previous kernel under PDL)
   if (t == 0) {
     for (int s = 0; s < stages; ++s) {
-      mbar_init(full0 + 8 * s, gather ? kEpiThreads + 1u : 1u);
+      mbar_init(full0 + 8 * s, gather ? kEpiThreadsPT + 1u : 1u);
       mbar_init(empty0 + 8 * s, 1u);
     }
     for (int j = 0; j < 2; ++j) {
       mbar_init(tfull0 + 8 * j, 1u);
-      mbar_init(tempty0 + 8 * j, static_cast<uint32_t>(kEpiThreads));
+      mbar_init(tempty0 + 8 * j, static_cast<uint32_t>(kEpiThreadsPT));
       mbar_init(res0 + 8 * j, 1u);
-      mbar_init(staged0 + 8 * j, static_cast<uint32_t>(kEpiThreads));
+      mbar_init(staged0 + 8 * j, static_cast<uint32_t>(kEpiThreadsPT));
       mbar_init(rofree0 + 8 * j, 1u);
     }
     mbar_init(recv_bar, 1u);
@@ -720,13 +720,13 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
     }
     fence_barrier_init();
   }
-  if (warp == kEpiWarps && lane == 0) {
+  if (warp == kEpiWarpsPT && lane == 0) {
     if (!gather) tma_prefetch_desc(&p.tmap_a);
     tma_prefetch_desc(&p.tmap_b);
     if (p.c_tma) tma_prefetch_desc(&p.tmap_c);
     if (res_tma) tma_prefetch_desc(&p.tmap_r);
   }
-  if (warp == kEpiWarps + 1) tmem_alloc(smem_u32(tmem_slot), p.tmem_cols);
+  if (warp == kEpiWarpsPT + 1) tmem_alloc(smem_u32(tmem_slot), p.tmem_cols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -738,7 +738,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
   // griddepcontrol.wait is per role: weights (B, bias) do not depend on the
   // previous layer, so they are fetched before it; activations after it.
 
-  if (warp == kEpiWarps) {
+  if (warp == kEpiWarpsPT) {
     // ================= TMA producer
     if (lane == 0) {
       int s = 0;
@@ -824,7 +824,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
       }
     }
     __syncwarp();
-  } else if (kPersistent && warp == kEpiWarps + 2) {
+  } else if (kPersistent && warp == kEpiWarpsPT + 2) {
     if (lane == 0 && p.c_tma) {
       // ================= store agent: TMA-stores each staged output tile, frees the
       // staging buffer, and loads the residual tile two tiles ahead into it, so no
@@ -864,7 +864,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
       }
     }
     __syncwarp();
-  } else if (warp == kEpiWarps + 1) {
+  } else if (warp == kEpiWarpsPT + 1) {
     // ================= MMA issuer (one thread issues for the whole CTA)
     if (lane == 0) {
       int s = 0;
@@ -935,7 +935,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
       }
       if (kAllowGather && gather) {
         // implicit im2col: thread t owns 16 B chunk j = t % 8 of rows rg + kGR * ri
-        constexpr int kGR = kEpiThreads / 8;  // rows per pass
+        constexpr int kGR = kEpiThreadsPT / 8;  // rows per pass
         constexpr int kGI = kBM / kGR;        // passes per 128-row tile
         const int j = t & 7;
         const int rg = t >> 3;
@@ -1015,7 +1015,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           if (++gst_lag == stages) gst_lag = 0;
         }
       }
-      named_bar_sync(1, kEpiThreads);  // this tile's bias visible
+      named_bar_sync(1, kEpiThreadsPT);  // this tile's bias visible
       mbar_wait(tfull0 + 8 * buf, (it >> 1) & 1);
       tc_fence_after();
       if (kPersistent && p.c_tma) mbar_wait(rofree0 + 8 * buf, ((it >> 1) & 1) ^ 1);  // store of tile it-2 read it
@@ -1065,7 +1065,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           }
         }
         if (trace && t == 0) trace[4] = stamp();
-        named_bar_sync(1, kEpiThreads);  // own-slot rows visible to all epilogue threads
+        named_bar_sync(1, kEpiThreadsPT);  // own-slot rows visible to all epilogue threads
         mbar_wait(recv_bar, 0);          // every peer's rows have landed
         if (res_tma && slice_rows > 0) mbar_wait(res0 + 8 * buf, (it >> 1) & 1);
       } else {
@@ -1082,7 +1082,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
       //   splits  > 1: items (row, chunk) of this rank's slice, the S receive slots
       //                summed in fixed rank order 0..S-1 (deterministic)
       const int n_iter = splits == 1 ? (warp_live && half < cpr ? (cpr - half + 1) >> 1 : 0)
-                                     : max(0, (slice_rows * cpr - t + kEpiThreads - 1) / kEpiThreads);
+                                     : max(0, (slice_rows * cpr - t + kEpiThreadsPT - 1) / kEpiThreadsPT);
       for (int k = 0; k < n_iter; ++k) {
         float v[16];
         int row, cb;
@@ -1096,7 +1096,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           more = c + 2 < cpr;
           if (more) tmem_ld16_issue(taddr + (c + 2) * 16, r);
         } else {
-          const int item = t + k * kEpiThreads;
+          const int item = t + k * kEpiThreadsPT;
           const int lr = item / cpr;
           row = r0 + lr;
           cb = (item - lr * cpr) << 4;
@@ -1128,7 +1128,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
         if (kPersistent) {
           mbar_arrive(staged0 + 8 * buf);  // the store agent issues the TMA store
         } else {
-          named_bar_sync(1, kEpiThreads);
+          named_bar_sync(1, kEpiThreadsPT);
           if (t == 0 && slice_rows > 0) {
 #pragma unroll 1
             for (int j = 0; j < bn / box_cols; ++j)
@@ -1146,7 +1146,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
   // ---------------- teardown
   tc_fence_before();
   __syncthreads();
-  if (warp == kEpiWarps + 1) {
+  if (warp == kEpiWarpsPT + 1) {
     tc_fence_after();
     tmem_dealloc(tmem_base, p.tmem_cols);
   }

@@ -10,10 +10,21 @@ namespace pask {
 
 constexpr int kBM = 128;       // UMMA M (cta_group::1): one TMEM lane per tile row
 constexpr int kBK = 64;        // 64 bf16 = 128 B = one SWIZZLE_128B row
-constexpr int kEpiWarps = 8;       // warps 0-7: bias, gather (A_GATHER), epilogue
+#ifndef PASK_EPI_WARPS
+#define PASK_EPI_WARPS 8
+#endif
+// one-tile contraction kernel: warps 0..kEpiWarps-1 load the bias, gather
+// (A_GATHER) and run the epilogue, kEpiGroups warps per TMEM lane quarter
+constexpr int kEpiWarps = PASK_EPI_WARPS;
+static_assert(kEpiWarps % 4 == 0, "epilogue warps cover the four TMEM lane quarters");
+constexpr int kEpiGroups = kEpiWarps / 4;
 constexpr int kEpiThreads = 32 * kEpiWarps;
-constexpr int kGemmThreads = kEpiThreads + 64;    // + warp 8 TMA producer, warp 9 TMEM + MMA
-constexpr int kGemmThreadsPT = kEpiThreads + 96;  // persistent: + warp 10 store / residual agent
+constexpr int kGemmThreads = kEpiThreads + 64;  // + TMA producer warp, TMEM / MMA warp
+// persistent-tile kernel: 8 epilogue warps (its 157 registers per thread do not
+// fit more), + TMA producer, TMEM / MMA and store / residual agent warps
+constexpr int kEpiWarpsPT = 8;
+constexpr int kEpiThreadsPT = 32 * kEpiWarpsPT;
+constexpr int kGemmThreadsPT = kEpiThreadsPT + 96;
 
 // A-operand source of the contraction kernel.
 enum AMode : int32_t {
