@@ -170,6 +170,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   constexpr uint32_t kABytes = kBM * kBK * 2;  // 16 KB
   const uint32_t b_bytes = static_cast<uint32_t>(bn) * kBK * 2;
   const uint32_t stage_bytes = kABytes + b_bytes;
+  const uint32_t a_tx = static_cast<uint32_t>(p.a_rows) * (kBK * 2);  // A bytes a TMA k-block delivers
   // ---- smem carve-up (mirrors gemm_tiling() on the host)
   const uint32_t ring_bytes = (stages * stage_bytes + 1023u) & ~1023u;
   const uint32_t recv_pitch = (bn + 4) * 4;  // fp32 split-K receive row pitch (bank spread)
@@ -281,7 +282,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       for (int i = 0; i < pre; ++i) {
         const uint32_t sb = smem_base + i * stage_bytes + kABytes;
         const int kb = kb_begin + i;
-        mbar_arrive_expect_tx(full0 + 8 * i, b_bytes + (gather ? 0u : kABytes));
+        mbar_arrive_expect_tx(full0 + 8 * i, b_bytes + (gather ? 0u : a_tx));
         if (p.b_major == 0) {
           tma_load_3d(sb, &p.tmap_b, full0 + 8 * i, kb * kBK, n0, b);
         } else {
@@ -307,7 +308,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const uint32_t sa = smem_base + s * stage_bytes;
         const uint32_t sb = sa + kABytes;
         const int kb = kb_begin + i;
-        if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
+        if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : a_tx));
         if (kAllowGather && im2col) {
           tma_load_im2col_4d(sa, &p.tmap_a, full0 + 8 * s, cc * 64, iw, ih, in,
                              static_cast<uint16_t>(ts * gDW), static_cast<uint16_t>(tr * gDH));
@@ -409,7 +410,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       int c = kk - tap * gC;
       int r = tap / gS;
       int s = tap - r * gS;
-      const int lag = min(2, stages - 1);
+      const int lag = min(p.gather_lag, stages - 1);  // k-blocks of cp.async in flight before publishing
       int st = 0, st_lag = 0;  // ring slot being filled / being published
       uint32_t ph = 0;
       for (int i = 0; i < nk; ++i) {
@@ -911,7 +912,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
     const int erow = quarter * 32 + lane;  // tile row == TMEM lane read by this thread
     const int cpr = bn >> 4;                // 16-column chunks per row
     // gather ring position (persists across tiles)
-    const int lag = min(2, stages - 1);
+    const int lag = min(p.gather_lag, stages - 1);
     int gst = 0, gst_lag = 0;
     uint32_t gph = 0;
     for (int tile = tile0, it = 0; tile < n_tiles_total; tile += tstep, ++it) {

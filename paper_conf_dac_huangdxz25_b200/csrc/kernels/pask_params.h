@@ -62,6 +62,10 @@ struct alignas(64) GemmParams {
   int32_t m_tiles, n_tiles;
   int32_t c_tma;         // 1: output (and residual) through TMA + smem staging
   int32_t rows_per;      // rows reduced / stored per cluster rank = 128 / splits
+  int32_t gather_lag;    // A_GATHER: k-blocks of cp.async kept in flight before a slot is published
+  int32_t a_rows;        // A rows TMA-loaded per k-block: 128, or 64 when the whole M fits
+                         // in 64 rows (one m-tile; rows 64-127 of the operand are never
+                         // stored, so their stale smem contents only reach unread TMEM lanes)
   // implicit-GEMM geometry (A_GATHER): input [n][H][W][C], output pixel m -> (n, p, q)
   int32_t H, W, C, P, Q, R, S;
   int32_t sh, sw, ph, pw, dh, dw;
