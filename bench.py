@@ -187,6 +187,9 @@ def main():
     ap.add_argument("--model", default="resnet50",
                     choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base", "bert_base_fa"])
     ap.add_argument("--batch", type=int, default=1, help="images per inference (Table II sweep)")
+    ap.add_argument("--branches", type=int, default=1, choices=[0, 1],
+                    help="1 (default): independent nodes (ResNet downsample convs) on a second stream in "
+                         "the hot graph (DESIGN.md D9)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cold-samples", type=int, default=4,
                     help="extra fresh-process cold starts (N = 1); cold_over_hot uses the median")
@@ -245,7 +248,7 @@ def main():
 
     flush()
     torch.cuda.synchronize()
-    ctx = P.Context(local_rank, P.config(packaging=args.packaging, graph=args.graph))
+    ctx = P.Context(local_rank, P.config(packaging=args.packaging, graph=args.graph, branches=args.branches))
     n_nodes = len(spec["layers"])
 
     def barrier():
@@ -420,6 +423,8 @@ def main():
                    "parallelism": f"replicas{world}",
                    "packaging": ["one code object per kernel", "single code object",
                                  "operator families (memory-bound + contraction)"][args.packaging],
+                   "branches": "independent nodes on a second stream in the hot graph" if args.branches
+                               else "one stream",
                    "hot_issue": "CUDA graph replay (captured on the 2nd inference)" if args.graph
                                 else "direct cuLaunchKernelEx per layer",
                    "l2": "warm (no flush)" if args.no_flush else

@@ -213,6 +213,12 @@ typedef struct {
   int32_t catalog;    /* 0 = generic catalog; 1 = tuned catalog: s* of a dense conv is its
                          per-problem specialised solution when one exists (the library
                          behaviour PASK starts from; the Baseline scheme)       */
+  int32_t branches;   /* 1 = a node that does not read its predecessor's output (ResNet's
+                         downsample conv) runs on a second stream, forked after its last
+                         producer and joined before its first consumer, so it overlaps the
+                         main chain (D9); 0 = one stream, node order.  Ignored
+                         with instrument = 1.  Same kernels and parameters either way:
+                         outputs are bitwise identical                                       */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;

@@ -29,8 +29,9 @@ extern "C" {
 int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail_kernel);
 
 /* The fake driver's event log since the last enable: out[i] = kernel id of
- * the i-th event, kinds[i] = 0 for a completed load, 1 for a launch, 2 for a
- * launch of a kernel that was not yet loaded (must never happen).  Under
+ * the i-th event, kinds[i] = 0 for a completed load, 1 for a launch on the
+ * caller's stream, 3 for a launch on another stream (pask_config.branches), 2
+ * for a launch of a kernel that was not yet loaded (must never happen).  Under
  * packaging 2 the `pask_mem` family entry logs as id PASK_MAX_KERNELS - 1 and
  * the contraction family as PASK_K_CONV_IGEMM.  Returns the number of events
  * (writes at most cap). */

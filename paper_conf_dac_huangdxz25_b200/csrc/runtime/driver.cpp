@@ -63,6 +63,7 @@ void resolve() {
   PASK_RESOLVE(cuStreamSynchronize)
   PASK_RESOLVE(cuStreamCreate)
   PASK_RESOLVE(cuStreamDestroy)
+  PASK_RESOLVE(cuStreamWaitEvent)
   PASK_RESOLVE(cuStreamBeginCapture)
   PASK_RESOLVE(cuStreamEndCapture)
   PASK_RESOLVE(cuGraphInstantiateWithFlags)

@@ -37,6 +37,7 @@ struct Driver {
   PASK_DRV_FN(cuStreamSynchronize)
   PASK_DRV_FN(cuStreamCreate)
   PASK_DRV_FN(cuStreamDestroy)
+  PASK_DRV_FN(cuStreamWaitEvent)
   PASK_DRV_FN(cuStreamBeginCapture)
   PASK_DRV_FN(cuStreamEndCapture)
   PASK_DRV_FN(cuGraphInstantiateWithFlags)

@@ -5,6 +5,7 @@
 #include <string.h>
 
 #include <chrono>
+#include <atomic>
 #include <mutex>
 #include <thread>
 #include <vector>
@@ -96,14 +97,17 @@ CUresult f_func_is_loaded(CUfunctionLoadingState* s, CUfunction f) {
   return CUDA_SUCCESS;
 }
 CUresult f_func_set_attr(CUfunction, CUfunction_attribute, int) { return CUDA_SUCCESS; }
-CUresult f_launch(const CUlaunchConfig*, CUfunction f, void**, void**) {
+CUresult f_launch(const CUlaunchConfig* cfg, CUfunction f, void**, void**) {
   const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
   bool loaded;
   {
     std::lock_guard<std::mutex> lk(g_mu);
     loaded = id >= 0 && id < PASK_MAX_KERNELS && g_loaded[id];
   }
-  log_event(id, loaded ? 1 : 2);
+  // 1: launch on the caller's stream, 3: on another stream (the branches side
+  // stream, D9), 2: kernel not loaded (must never happen)
+  const uintptr_t sh = reinterpret_cast<uintptr_t>(cfg->hStream);
+  log_event(id, !loaded ? 2 : (sh <= 0x40 ? 1 : 3));
   return CUDA_SUCCESS;
 }
 CUresult f_tmap_tiled(CUtensorMap* m, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
@@ -132,12 +136,30 @@ CUresult f_event_elapsed(float* ms, CUevent, CUevent) {
 CUresult f_h2d(CUdeviceptr, const void*, size_t, CUstream) { return CUDA_SUCCESS; }
 CUresult f_d2h(void*, CUdeviceptr, size_t, CUstream) { return CUDA_SUCCESS; }
 CUresult f_stream_sync(CUstream) { return CUDA_SUCCESS; }
+// streams get handles 0x40, 0x41, ... in creation order: the caller's stream
+// (0) and the first created one (the graph-capture stream) are "main", later
+// ones (the branches side stream) are logged as kind 3
+std::atomic<uintptr_t> g_next_stream{0x40};
 CUresult f_stream_create(CUstream* s, unsigned int) {
-  *s = fake_handle<CUstream>(0x40);
+  *s = fake_handle<CUstream>(g_next_stream.fetch_add(1));
   return CUDA_SUCCESS;
 }
 CUresult f_stream_destroy(CUstream) { return CUDA_SUCCESS; }
-CUresult f_begin_capture(CUstream, CUstreamCaptureMode) { return CUDA_ERROR_NOT_SUPPORTED; }
+// graph capture: launches during a capture are logged like direct launches (the
+// issue order is what the tests check); replaying the fake graph launches nothing
+CUresult f_begin_capture(CUstream, CUstreamCaptureMode) { return CUDA_SUCCESS; }
+CUresult f_end_capture(CUstream, CUgraph* g) {
+  *g = fake_handle<CUgraph>(0x50);
+  return CUDA_SUCCESS;
+}
+CUresult f_graph_instantiate(CUgraphExec* ge, CUgraph, unsigned long long) {
+  *ge = fake_handle<CUgraphExec>(0x60);
+  return CUDA_SUCCESS;
+}
+CUresult f_graph_launch(CUgraphExec, CUstream) { return CUDA_SUCCESS; }
+CUresult f_graph_destroy(CUgraph) { return CUDA_SUCCESS; }
+CUresult f_graph_exec_destroy(CUgraphExec) { return CUDA_SUCCESS; }
+CUresult f_stream_wait_event(CUstream, CUevent, unsigned int) { return CUDA_SUCCESS; }
 
 Driver make_fake() {
   Driver d;
@@ -167,6 +189,12 @@ Driver make_fake() {
   d.cuStreamCreate = f_stream_create;
   d.cuStreamDestroy = f_stream_destroy;
   d.cuStreamBeginCapture = f_begin_capture;
+  d.cuStreamEndCapture = f_end_capture;
+  d.cuGraphInstantiateWithFlags = f_graph_instantiate;
+  d.cuGraphLaunch = f_graph_launch;
+  d.cuGraphDestroy = f_graph_destroy;
+  d.cuGraphExecDestroy = f_graph_exec_destroy;
+  d.cuStreamWaitEvent = f_stream_wait_event;
   d.ok = true;
   return d;
 }
@@ -183,6 +211,7 @@ PASK_API int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail
   g_ids.clear();
   g_kinds.clear();
   memset(g_loaded, 0, sizeof(g_loaded));
+  g_next_stream.store(0x40);
   if (enable) {
     g_fake = make_fake();
     driver_override(&g_fake);

@@ -57,7 +57,7 @@ class Config(C.Structure):
     _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
                 ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
                 ("packaging", C.c_int32), ("interleave", C.c_int32), ("graph", C.c_int32),
-                ("catalog", C.c_int32)]
+                ("catalog", C.c_int32), ("branches", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -154,9 +154,9 @@ def function_name(k, packaging):
 
 
 def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,
-           interleave=0, graph=0, catalog=0):
+           interleave=0, graph=0, catalog=0, branches=0):
     return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph,
-                  catalog)
+                  catalog, branches)
 
 
 def test_fake_driver(enable=True, load_us=0, fail_kernel=-1):

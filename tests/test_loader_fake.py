@@ -179,3 +179,57 @@ def test_promote_loads_skipped_solutions_in_order():
     n_tuned = ctx.promote(target_catalog=1)
     assert n_tuned == 53                                           # every conv -> its specialisation
     ctx.close()
+
+
+def expected_side_nodes(spec):
+    """Restatement of the branches rule (D9): node i goes to the side
+    stream when it reads an earlier node's output but not node i-1's (its last
+    producer is before i-1), and none of its producers is itself a side node."""
+    producer, side = {}, []
+    for i, L in enumerate(spec["layers"]):
+        srcs = [t for t in list(L["inputs"]) + ([L["res"]] if L.get("res") else []) if t in producer]
+        if srcs:
+            prod = max(producer[t] for t in srcs)
+            if prod < i - 1 and not any(producer[t] in side for t in srcs):
+                side.append(i)
+        producer[L["out"]] = i
+    return side
+
+
+@pytest.mark.parametrize("name", ["resnet50", "mobilenet_v2", "bert_base", "tiny_cnn"])
+def test_branches_issue_side_nodes_after_their_producer(name):
+    """cfg.branches: in the captured hot graph the side nodes (ResNet-50's four
+    downsample convs; none in the other configs) launch on the second stream
+    right after their last producer, everything else on the main stream in node
+    order; the cold direct issue stays on one stream in node order."""
+    spec, _ = build_model(name)
+    dm = DeviceModel(spec, alloc=False)
+    P.test_fake_driver(True, load_us=0)
+    ctx = P.Context(0, P.config(branches=1, graph=1))
+    plan = ctx.load_model(dm.graph)
+    for _ in range(3):   # cold direct issue, then capture (2nd call), then a replay
+        ctx.infer(0)
+    ctx.sync()
+    ctx.close()
+    log = [(k, kind) for k, kind in P.test_fake_log() if kind != 0]
+    n = len(spec["layers"])
+    assert len(log) == 2 * n                      # the replay launches nothing in the fake
+    assert log[:n] == [(b[2], 1) for b in plan]   # cold: one stream, node order
+    launches = log[n:]                            # the captured sequence
+    side = expected_side_nodes(spec)
+    assert len(side) == (4 if name == "resnet50" else 0)
+    # expected issue order: main nodes in order, each side node right after its producer
+    producer = {L["out"]: i for i, L in enumerate(spec["layers"])}
+    order = []
+    for i, L in enumerate(spec["layers"]):
+        if i in side:
+            continue
+        order.append((i, 1))
+        for j in side:
+            srcs = [t for t in list(spec["layers"][j]["inputs"]) +
+                    ([spec["layers"][j]["res"]] if spec["layers"][j].get("res") else []) if t in producer]
+            if max(producer[t] for t in srcs) == i:
+                order.append((j, 3))
+    bound = [b[2] for b in plan]
+    assert [(k, kind) for k, kind in launches] == [(bound[i], kind) for i, kind in order]
+    assert sum(1 for _, kind in launches if kind == 3) == len(side)
