@@ -1,4 +1,4 @@
-"""Debug: GPU timeline of one hot inference (PDL on, direct issue): per
+"""Debug: GPU timeline of one hot inference (PDL on, graph replay as bench.py): per
 contraction node, first CTA start / last CTA end and median phase times."""
 import os
 import sys
@@ -23,7 +23,8 @@ n = len(spec["layers"])
 buf = torch.zeros(n * 8 * 4096, dtype=torch.int64, device="cuda")
 os.environ["PASK_TRACE_NODE"] = "-1"
 os.environ["PASK_TRACE_PTR"] = str(buf.data_ptr())
-ctx = P.Context(0, P.config())
+# the bench configuration: families packaging, hot graph with branches
+ctx = P.Context(0, P.config(packaging=2, graph=1, branches=1))
 ctx.load_model(dm.graph)
 s = torch.cuda.current_stream().cuda_stream
 for _ in range(5):
