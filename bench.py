@@ -196,9 +196,9 @@ def main():
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
                     help="1: hot inferences replay a CUDA graph captured on the 2nd call")
-    ap.add_argument("--packaging", type=int, default=2, choices=[0, 1, 2],
+    ap.add_argument("--packaging", type=int, default=2, choices=[0, 1, 2, 3],
                     help="0: one code object per catalog kernel; 1: whole catalog in one; "
-                         "2 (default): operator families, DESIGN.md D8")
+                         "2 (default): operator families, DESIGN.md D8; 3: single function, D10")
     args = ap.parse_args()
     args.workload_name = {
         "tiny_cnn": "tiny CNN 3xconv3x3(16/32/64)+maxpool+FC, 32x32x3, batch 1, bf16",
@@ -386,7 +386,7 @@ def main():
     # replicas the ranks' own cold starts are the concurrent measurement)
     fresh = []
     if args.cold_samples > 0 and world == 1:
-        scheme = ["pask", "pask_single_image", "pask_families"][args.packaging]
+        scheme = ["pask", "pask_single_image", "pask_families", "pask_single_function"][args.packaging]
         for _ in range(args.cold_samples):
             r = subprocess.run([sys.executable, os.path.join(ROOT, "scripts", "cold_samples.py"), "--model",
                                 args.model, "--child", scheme, "--batch", str(args.batch)],
@@ -422,7 +422,8 @@ def main():
                    "global_batch": world * args.batch, "per_gpu_batch": args.batch,
                    "parallelism": f"replicas{world}",
                    "packaging": ["one code object per kernel", "single code object",
-                                 "operator families (memory-bound + contraction)"][args.packaging],
+                                 "operator families (memory-bound + contraction)",
+                                 "single function (both families behind one entry)"][args.packaging],
                    "branches": "independent nodes on a second stream in the hot graph" if args.branches
                                else "one stream",
                    "hot_issue": "CUDA graph replay (captured on the 2nd inference)" if args.graph

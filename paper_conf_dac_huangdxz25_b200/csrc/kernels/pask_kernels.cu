@@ -9,6 +9,25 @@
 
 using namespace pask;
 
+// PASK_MEM_MASK (bit per MemKind) drops memory-family cases at compile time
+// (upload-size experiments only; the shipped families carry every case).
+#ifndef PASK_MEM_MASK
+#define PASK_MEM_MASK 0x3f
+#endif
+#define PASK_MEM_HAS(k) ((PASK_MEM_MASK >> (k)) & 1)
+
+// The memory-bound family: the solution's own body selected by p.kind.
+__device__ __forceinline__ void mem_dispatch(const MemParams& p) {
+  switch (p.kind) {
+    case MEM_LAYOUT: if (PASK_MEM_HAS(MEM_LAYOUT)) layout_body(p.l); break;
+    case MEM_DW: if (PASK_MEM_HAS(MEM_DW)) dw_body(p.d); break;
+    case MEM_POOL: if (PASK_MEM_HAS(MEM_POOL)) pool_body(p.p); break;
+    case MEM_GAVG: if (PASK_MEM_HAS(MEM_GAVG)) gavg_body(p.p); break;
+    case MEM_SOFTMAX: if (PASK_MEM_HAS(MEM_SOFTMAX)) softmax_body(p.r); break;
+    default: if (PASK_MEM_HAS(MEM_LAYERNORM)) layernorm_body(p.r); break;
+  }
+}
+
 extern "C" {
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_layout
@@ -84,15 +103,19 @@ __global__ void __launch_bounds__(256) pask_layernorm(const __grid_constant__ Ro
 // CUfunction -- one code upload instead of up to six (a function upload costs a
 // fixed ~20-40 us on top of its size, profiles/r01_loader_microbench.md).  Each
 // case is the same body as the solution's own entry, so outputs are bitwise equal.
-__global__ void __launch_bounds__(256) pask_mem(const __grid_constant__ MemParams p) {
-  switch (p.kind) {
-    case MEM_LAYOUT: layout_body(p.l); break;
-    case MEM_DW: dw_body(p.d); break;
-    case MEM_POOL: pool_body(p.p); break;
-    case MEM_GAVG: gavg_body(p.p); break;
-    case MEM_SOFTMAX: softmax_body(p.r); break;
-    default: layernorm_body(p.r); break;
-  }
+__global__ void __launch_bounds__(256) pask_mem(const __grid_constant__ MemParams p) { mem_dispatch(p); }
+#endif
+
+#if defined(PASK_ONLY_KERNEL) && PASK_ONLY_KERNEL_pask_all  // own code object only
+// Single-function entry of packaging 3 (D10): the generic contraction
+// body and the memory family behind one branch on a uniform parameter -- one code
+// upload for a whole CNN / transformer catalog.  Same bodies as the solutions' own
+// entries, so outputs are bitwise equal.
+__global__ void __launch_bounds__(kGemmThreads, 1) pask_all(const __grid_constant__ AllParams p) {
+  if (p.g.family == 0)
+    conv_gemm_body<true>(p.g);
+  else
+    mem_dispatch(p.m);
 }
 #endif
 

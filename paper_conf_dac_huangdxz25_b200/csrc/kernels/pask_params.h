@@ -4,6 +4,7 @@
 // at pask_load_model time (overlapping the proactive loads).
 #pragma once
 #include <cuda.h>
+#include <stddef.h>
 #include <stdint.h>
 
 namespace pask {
@@ -72,6 +73,7 @@ struct alignas(64) GemmParams {
   uint32_t idesc;      // tcgen05 instruction descriptor (kind::f16, bf16 x bf16 -> f32)
   uint32_t tmem_cols;  // power of two >= max(32, bn)
   uint32_t smem_bytes;
+  int32_t family;      // pask_all (packaging 3): 0 = this block, 1 = the MemParams overlaid at offset 0
 };
 
 struct alignas(16) LayoutParams {
@@ -136,5 +138,16 @@ struct alignas(16) MemParams {
   };
   int32_t kind;  // MemKind
 };
+
+// Single-function entry (pask_config.packaging = 3): the contraction body and the
+// memory-bound family in ONE CUfunction, `pask_all`, so a model's whole catalog
+// becomes resident with one code upload.  g.family 0 runs g, 1 runs m (m lies at
+// offset 0, below g.family, so a contraction launch passes the same bytes as in
+// the other packagings).
+union alignas(64) AllParams {
+  GemmParams g;
+  MemParams m;
+};
+static_assert(sizeof(MemParams) <= offsetof(GemmParams, family), "family flag outside the memory block");
 
 }  // namespace pask

@@ -25,11 +25,13 @@ int g_fail_kernel = -1;
 std::vector<int32_t> g_ids, g_kinds;
 bool g_loaded[PASK_MAX_KERNELS] = {};
 constexpr int32_t kFakeMemFamilyId = PASK_MAX_KERNELS - 1;  // id logged for the `pask_mem` entry
+constexpr int32_t kFakeAllId = PASK_MAX_KERNELS - 2;        // id logged for the `pask_all` entry
 
 int32_t kernel_of_name(const char* name) {
   for (int32_t k = 0; k < num_kernels(); ++k)
     if (strcmp(catalog(k).name, name) == 0) return k;
   if (strcmp(name, "pask_mem") == 0) return kFakeMemFamilyId;  // packaging-2 family entry
+  if (strcmp(name, "pask_all") == 0) return kFakeAllId;        // packaging-3 single entry
   return -1;
 }
 void sleep_us(int us) {

@@ -26,6 +26,7 @@ SCHEMES = {
     "pask_interleave": dict(proactive=1, interleave=1),  # Fig. 5 interleaving
     "pask_single_image": dict(packaging=1),           # whole catalog as one code object
     "pask_families": dict(packaging=2),               # operator families (D8)
+    "pask_single_function": dict(packaging=3),        # both families in one CUfunction (D10)
     "pask_i": dict(reuse=0),                          # PaSK-I: proactive, no reuse
     "pask_r": dict(search=1),                         # PaSK-R: naive (exhaustive-order) search
     "reactive": dict(proactive=0, reuse=0),           # Baseline analog: lazy load at first launch

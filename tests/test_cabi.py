@@ -191,4 +191,5 @@ def test_kernel_function_families():
         assert P.function_name(k, 0) == P.function_name(k, 1) == P.kernel_name(k)
         want = "pask_mem" if k in mem else "pask_conv_igemm" if k in contract else P.kernel_name(k)
         assert P.function_name(k, 2) == want
+        assert P.function_name(k, 3) == ("pask_all" if k in mem | contract else P.kernel_name(k))
     assert P.function_name(-1, 2) == "" and P.function_name(P.num_kernels(), 0) == ""

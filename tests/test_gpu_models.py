@@ -83,7 +83,7 @@ def test_tuned_catalog_specialised_kernels(name):
     ctx2.close()
 
 
-@pytest.mark.parametrize("packaging", [0, 1, 2])
+@pytest.mark.parametrize("packaging", [0, 1, 2, 3])
 @pytest.mark.parametrize("cfg", ["reactive", "pask_i", "pask_r", "no_pdl"])
 def test_schemes_same_outputs(cfg, packaging):
     """Every scheme of PAPER.md:174-186 (reactive loading, PaSK-I = no reuse,
@@ -108,6 +108,8 @@ def test_schemes_same_outputs(cfg, packaging):
     st = ctx.stats()
     if packaging == 2:   # ResNet-50's solutions fall in two families, one code object
         assert st["kernels_loaded"] == 2 and st["code_objects_loaded"] == 1
+    elif packaging == 3:  # ... and in one function under packaging 3
+        assert st["kernels_loaded"] == 1 and st["code_objects_loaded"] == 1
     else:
         assert st["kernels_loaded"] == len(o["loaded"])
         assert st["code_objects_loaded"] == (1 if packaging == 1 else len(o["loaded"]))
@@ -136,6 +138,31 @@ def test_family_packaging_bitwise(name):
     dm2, ctx2, _ = run_model(spec, x)
     for L in spec["layers"]:
         np.testing.assert_array_equal(fam_out[L["out"]], dm2.read_raw(L["out"]))
+    ctx2.close()
+
+
+@pytest.mark.parametrize("name", MODELS)
+def test_single_function_packaging_bitwise(name):
+    """Packaging 3 (D10): the same plan as packaging 0, every
+    contraction and memory-bound solution served by the one `pask_all` upload
+    (attention keeps its own object), and every layer's output bitwise equal to
+    the per-kernel code objects' (same bodies, same parameters)."""
+    spec, x = build_model(name)
+    dm, ctx, plan = run_model(spec, x, cfg=P.config(packaging=3))
+    o = OP.execution_plan(OP.problems_from_spec(spec))
+    assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
+    st = ctx.stats()
+    fam = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM,
+           P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
+    own = set(o["loaded"]) - fam
+    assert st["kernels_loaded"] == len(own) + 1
+    assert st["code_objects_loaded"] == len(own) + 1
+    assert {k for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k)} >= set(o["loaded"])
+    one_out = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
+    ctx.close()
+    dm2, ctx2, _ = run_model(spec, x)
+    for L in spec["layers"]:
+        np.testing.assert_array_equal(one_out[L["out"]], dm2.read_raw(L["out"]))
     ctx2.close()
 
 

@@ -32,16 +32,20 @@ MODES = [
     dict(proactive=2, packaging=1), dict(proactive=2, reuse=0), dict(proactive=1, search=1),
     dict(proactive=0, reuse=0, catalog=1), dict(proactive=2, catalog=1),
     dict(proactive=2, packaging=2), dict(proactive=1, packaging=2), dict(proactive=0, packaging=2),
+    dict(proactive=2, packaging=3), dict(proactive=1, packaging=3), dict(proactive=0, packaging=3),
 ]
 
 # packaging 2 (D8): the CUfunction that serves a catalog solution, as
 # the fake driver logs it (the memory family entry `pask_mem` is id 63)
 FAM_MEM = 63
+FAM_ALL = 62   # packaging 3 (D10): `pask_all`
 MEM_SOLUTIONS = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM}
 CONTRACT_SOLUTIONS = {P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
 
 
 def function_of(k, packaging):
+    if packaging == 3:
+        return FAM_ALL if k in MEM_SOLUTIONS | CONTRACT_SOLUTIONS else k
     if packaging != 2:
         return k
     if k in MEM_SOLUTIONS:
