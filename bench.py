@@ -387,6 +387,8 @@ def main():
     fresh = []
     if args.cold_samples > 0 and world == 1:
         scheme = ["pask", "pask_single_image", "pask_families", "pask_single_function"][args.packaging]
+        if args.branches and args.packaging == 2:
+            scheme = "pask_families_branches"  # the same pask_config as this process's context
         for _ in range(args.cold_samples):
             r = subprocess.run([sys.executable, os.path.join(ROOT, "scripts", "cold_samples.py"), "--model",
                                 args.model, "--child", scheme, "--batch", str(args.batch)],

@@ -98,10 +98,24 @@ __device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint3
       }
     }
     act16(v, p.act);
-    sts_u4(a0, pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
-           pack_bf16x2(v[6], v[7]));
-    sts_u4(a1, pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
-           pack_bf16x2(v[14], v[15]));
+    const uint4 w0 = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                                pack_bf16x2(v[6], v[7]));
+    const uint4 w1 = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
+                                pack_bf16x2(v[14], v[15]));
+    if (p.c_tma == 2) {
+      // direct epilogue: 32 B of one output row straight from registers (N % 16 == 0,
+      // 16-byte aligned rows; the host picks it for the one-tile kernel only)
+      if (n0 + cb < p.N) {
+        uint4* o = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + p.off_c +
+                                            static_cast<int64_t>(b) * p.stride_c +
+                                            static_cast<int64_t>(m0 + row) * p.ldc + n0 + cb);
+        o[0] = w0;
+        o[1] = w1;
+      }
+      return;
+    }
+    sts_u4(a0, w0.x, w0.y, w0.z, w0.w);
+    sts_u4(a1, w1.x, w1.y, w1.z, w1.w);
     return;
   }
   // unaligned output rows (e.g. N = 10): scalar stores, residual from global
@@ -566,7 +580,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       if (more) tmem_ld_wait(r);
     }
     if (trace && t == 0) trace[6] = stamp();
-    if (p.c_tma) {
+    if (p.c_tma == 1) {
       fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
       named_bar_sync(1, kEpiThreads);
       if (t == 0 && slice_rows > 0) {

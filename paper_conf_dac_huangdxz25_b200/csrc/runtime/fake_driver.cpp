@@ -99,6 +99,8 @@ CUresult f_func_is_loaded(CUfunctionLoadingState* s, CUfunction f) {
   return CUDA_SUCCESS;
 }
 CUresult f_func_set_attr(CUfunction, CUfunction_attribute, int) { return CUDA_SUCCESS; }
+// the stream the last capture began on: "main" like the caller's stream (0)
+std::atomic<uintptr_t> g_capture_stream{0};
 CUresult f_launch(const CUlaunchConfig* cfg, CUfunction f, void**, void**) {
   const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
   bool loaded;
@@ -109,7 +111,8 @@ CUresult f_launch(const CUlaunchConfig* cfg, CUfunction f, void**, void**) {
   // 1: launch on the caller's stream, 3: on another stream (the branches side
   // stream, D9), 2: kernel not loaded (must never happen)
   const uintptr_t sh = reinterpret_cast<uintptr_t>(cfg->hStream);
-  log_event(id, !loaded ? 2 : (sh <= 0x40 ? 1 : 3));
+  const bool main_stream = sh == 0 || sh == g_capture_stream.load();
+  log_event(id, !loaded ? 2 : (main_stream ? 1 : 3));
   return CUDA_SUCCESS;
 }
 CUresult f_tmap_tiled(CUtensorMap* m, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
@@ -138,9 +141,9 @@ CUresult f_event_elapsed(float* ms, CUevent, CUevent) {
 CUresult f_h2d(CUdeviceptr, const void*, size_t, CUstream) { return CUDA_SUCCESS; }
 CUresult f_d2h(void*, CUdeviceptr, size_t, CUstream) { return CUDA_SUCCESS; }
 CUresult f_stream_sync(CUstream) { return CUDA_SUCCESS; }
-// streams get handles 0x40, 0x41, ... in creation order: the caller's stream
-// (0) and the first created one (the graph-capture stream) are "main", later
-// ones (the branches side stream) are logged as kind 3
+// streams get handles 0x40, 0x41, ... in creation order; launches on the
+// caller's stream (0) or on the capture stream are "main" (kind 1), on any other
+// (the branches side streams) kind 3
 std::atomic<uintptr_t> g_next_stream{0x40};
 CUresult f_stream_create(CUstream* s, unsigned int) {
   *s = fake_handle<CUstream>(g_next_stream.fetch_add(1));
@@ -149,7 +152,10 @@ CUresult f_stream_create(CUstream* s, unsigned int) {
 CUresult f_stream_destroy(CUstream) { return CUDA_SUCCESS; }
 // graph capture: launches during a capture are logged like direct launches (the
 // issue order is what the tests check); replaying the fake graph launches nothing
-CUresult f_begin_capture(CUstream, CUstreamCaptureMode) { return CUDA_SUCCESS; }
+CUresult f_begin_capture(CUstream s, CUstreamCaptureMode) {
+  g_capture_stream.store(reinterpret_cast<uintptr_t>(s));
+  return CUDA_SUCCESS;
+}
 CUresult f_end_capture(CUstream, CUgraph* g) {
   *g = fake_handle<CUgraph>(0x50);
   return CUDA_SUCCESS;
@@ -214,6 +220,7 @@ PASK_API int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail
   g_kinds.clear();
   memset(g_loaded, 0, sizeof(g_loaded));
   g_next_stream.store(0x40);
+  g_capture_stream.store(0);
   if (enable) {
     g_fake = make_fake();
     driver_override(&g_fake);
