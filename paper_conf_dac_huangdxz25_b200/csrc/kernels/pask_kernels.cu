@@ -9,22 +9,29 @@
 
 using namespace pask;
 
-// PASK_MEM_MASK (bit per MemKind) drops memory-family cases at compile time
-// (upload-size experiments only; the shipped families carry every case).
+// PASK_MEM_MASK (bit per MemKind) selects the memory-family cases compiled into
+// a code object: packaging 2 ships the families object in variants (all cases,
+// CNN, CNN + depthwise, transformer) and loads the smallest one covering the
+// model's bound solutions (D8).  A case compiled out traps: the host
+// never binds it, and if it did the launch fails loudly instead of writing nothing.
 #ifndef PASK_MEM_MASK
 #define PASK_MEM_MASK 0x3f
 #endif
-#define PASK_MEM_HAS(k) ((PASK_MEM_MASK >> (k)) & 1)
+#define PASK_MEM_CASE(k, body) \
+  case k:                     \
+    if ((PASK_MEM_MASK >> (k)) & 1) { body; } else { __trap(); } \
+    break;
 
 // The memory-bound family: the solution's own body selected by p.kind.
 __device__ __forceinline__ void mem_dispatch(const MemParams& p) {
   switch (p.kind) {
-    case MEM_LAYOUT: if (PASK_MEM_HAS(MEM_LAYOUT)) layout_body(p.l); break;
-    case MEM_DW: if (PASK_MEM_HAS(MEM_DW)) dw_body(p.d); break;
-    case MEM_POOL: if (PASK_MEM_HAS(MEM_POOL)) pool_body(p.p); break;
-    case MEM_GAVG: if (PASK_MEM_HAS(MEM_GAVG)) gavg_body(p.p); break;
-    case MEM_SOFTMAX: if (PASK_MEM_HAS(MEM_SOFTMAX)) softmax_body(p.r); break;
-    default: if (PASK_MEM_HAS(MEM_LAYERNORM)) layernorm_body(p.r); break;
+    PASK_MEM_CASE(MEM_LAYOUT, layout_body(p.l))
+    PASK_MEM_CASE(MEM_DW, dw_body(p.d))
+    PASK_MEM_CASE(MEM_POOL, pool_body(p.p))
+    PASK_MEM_CASE(MEM_GAVG, gavg_body(p.p))
+    PASK_MEM_CASE(MEM_SOFTMAX, softmax_body(p.r))
+    PASK_MEM_CASE(MEM_LAYERNORM, layernorm_body(p.r))
+    default: __trap();
   }
 }
 

@@ -9,6 +9,7 @@ Checks, for every proactive / interleave / packaging / reuse mode:
 * a failed load propagates as PASK_ECUDA naming the kernel (no fallback);
 * nothing deadlocks (pytest-timeout), including destroy with pending loads.
 """
+import os
 import pytest
 
 from oracle import plan as OP
@@ -236,3 +237,33 @@ def test_branches_issue_side_nodes_after_their_producer(name):
     for launches in (log[:n], log[n:]):           # cold direct issue, then the captured sequence
         assert [(k, kind) for k, kind in launches] == [(bound[i], kind) for i, kind in order]
         assert sum(1 for _, kind in launches if kind == 3) == len(side)
+
+
+@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnn"), ("mobilenet_v2", "dw"),
+                                          ("bert_base", "tf"), ("bert_base_fa", "tf")])
+def test_family_variant_covers_the_plan(name, variant):
+    """Packaging 2 (D8): the families object is loaded in the smallest
+    variant whose memory-bound cases cover every solution the plan desires or
+    binds (CNN: layout / pool / global-average pool / softmax; + depthwise for
+    MobileNetV2; softmax / LayerNorm for BERT); one code object, whose bytes are
+    that variant's image (attention keeps its own object)."""
+    from paper_conf_dac_huangdxz25_b200 import build as B
+    spec, _ = build_model(name)
+    dm = DeviceModel(spec, alloc=False)
+    P.test_fake_driver(True, load_us=0)
+    ctx = P.Context(0, P.config(packaging=2))
+    plan = ctx.load_model(dm.graph)
+    ctx.infer(0)
+    ctx.sync()
+    st = ctx.stats()
+    ctx.close()
+    mask = B.FAMILY_VARIANTS[f"pask_families_{variant}"]
+    kinds = {P.K_LAYOUT: 0, P.K_CONV_DW: 1, P.K_POOL: 2, P.K_POOL_GAVG: 3, P.K_SOFTMAX: 4, P.K_LAYERNORM: 5}
+    need = {kinds[k] for b in plan for k in (b[1], b[2]) if k in kinds}
+    assert all((mask >> kd) & 1 for kd in need)
+    smaller = [m for v, m in B.FAMILY_VARIANTS.items() if bin(m).count("1") < bin(mask).count("1")]
+    assert not any(all((m >> kd) & 1 for kd in need) for m in smaller)   # no smaller variant covers it
+    own = [b[2] for b in plan if b[2] == P.K_ATTENTION][:1]
+    expect = os.path.getsize(os.path.join(B.BUILD, f"pask_families_{variant}.fatbin"))
+    expect += sum(os.path.getsize(os.path.join(B.BUILD, P.kernel_name(k) + ".fatbin")) for k in own)
+    assert st["code_bytes_loaded"] == expect
