@@ -71,10 +71,41 @@ __device__ __forceinline__ uint32_t ro_addr(uint32_t ro, int lb, int row, int co
 // box width of the staged epilogue for an N tile of bn columns (power of two)
 __device__ __forceinline__ int box_log2(int bn) { return bn >= 64 ? 6 : (bn == 32 ? 5 : 4); }
 
+// The parameters the epilogue reads, loaded by the epilogue warps while the
+// mainloop runs, so their first (cold constant-cache) reads are off the critical
+// path.  Measured: ResNet-50 hot 0.2872 -> 0.2854 ms.  The epilogue itself is
+// bound by TMEM reads (a 128 x 64 fp32 tile is 32 KB at 64 B/cycle per SM; the
+// first 16-column chunk lands ~750 cycles after the accumulator is ready even with
+// no epilogue math, DESIGN.md §6 K6).
+struct EpiArgs {
+  void* out;
+  const void* res;
+  int64_t ldc, off_c, stride_c;
+  int32_t M, N, act, c_tma;
+};
+__device__ __forceinline__ EpiArgs load_epi_args(const GemmParams& p) {
+  EpiArgs e;
+  e.out = p.out;
+  e.res = p.res;
+  e.ldc = p.ldc;
+  e.off_c = p.off_c;
+  e.stride_c = p.stride_c;
+  e.M = p.M;
+  e.N = p.N;
+  e.act = p.act;
+  e.c_tma = p.c_tma;
+  // consume the values here: the loads (and the constant-cache fills of their
+  // lines) happen now, not at the first chunk -- ptxas may still re-read the bank
+  // at the use sites, which then hit
+  asm volatile("" ::"l"(e.out), "l"(e.res), "l"(e.ldc), "l"(e.off_c), "l"(e.stride_c));
+  asm volatile("" ::"r"(e.M), "r"(e.N), "r"(e.act), "r"(e.c_tma));
+  return e;
+}
+
 // v = act(acc + bias + res) -> bf16 (RNE) for 16 columns [cb, cb+16) of tile row
-// `row`: staged in smem for the TMA tensor store (c_tma) or, for unaligned
-// output rows, stored directly.
-__device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint32_t ro, int lb, int m0,
+// `row`: staged in smem for the TMA tensor store (c_tma 1), stored straight from
+// registers (c_tma 2) or, for unaligned output rows, stored element by element.
+__device__ __forceinline__ void epi16(const EpiArgs& p, uint32_t sbias, uint32_t ro, int lb, int m0,
                                       int n0, int b, int row, int cb, float (&v)[16]) {
 #pragma unroll
   for (int q4 = 0; q4 < 4; ++q4) {
@@ -103,15 +134,12 @@ __device__ __forceinline__ void epi16(const GemmParams& p, uint32_t sbias, uint3
     const uint4 w1 = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
                                 pack_bf16x2(v[14], v[15]));
     if (p.c_tma == 2) {
-      // direct epilogue: 32 B of one output row straight from registers (N % 16 == 0,
-      // 16-byte aligned rows; the host picks it for the one-tile kernel only)
-      if (n0 + cb < p.N) {
-        uint4* o = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + p.off_c +
-                                            static_cast<int64_t>(b) * p.stride_c +
-                                            static_cast<int64_t>(m0 + row) * p.ldc + n0 + cb);
-        o[0] = w0;
-        o[1] = w1;
-      }
+      // direct epilogue: the 32 B of one output row in a single 256-bit store from
+      // registers (N % 16 == 0, 32-byte aligned rows; one-tile kernel only)
+      if (n0 + cb < p.N)
+        stg_u8(reinterpret_cast<__nv_bfloat16*>(p.out) + p.off_c + static_cast<int64_t>(b) * p.stride_c +
+                   static_cast<int64_t>(m0 + row) * p.ldc + n0 + cb,
+               w0, w1);
       return;
     }
     sts_u4(a0, w0.x, w0.y, w0.z, w0.w);
@@ -269,6 +297,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   pdl_launch_dependents();  // let the next layer's prologue start
   // griddepcontrol.wait is per role: weights (B, bias) do not depend on the
   // previous layer, so they are fetched before it; activations after it.
+  EpiArgs ea;  // epilogue warps: their parameters, in registers before the accumulator wait
 
   if (warp == kEpiWarps) {
     // ================= TMA producer
@@ -385,6 +414,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   } else {
     // ================= warps 0-7: bias, (gather), epilogue
     if (t < bn) s_bias[t] = (p.bias != nullptr && n0 + t < p.N) ? __ldg(p.bias + n0 + t) : 0.f;
+    ea = load_epi_args(p);
     pdl_wait();  // before reading this layer's activations (gather) or writing outputs
     if (kAllowGather && gather) {
       // implicit im2col: thread t owns 16 B chunk j = t % 8 of rows rg + kGR * ri
@@ -576,7 +606,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           }
         }
       }
-      if (erow < valid_rows) epi16(p, sbias, ro, lb, m0, n0, b, erow, cb, v);
+      if (erow < valid_rows) epi16(ea, sbias, ro, lb, m0, n0, b, erow, cb, v);
       if (more) tmem_ld_wait(r);
     }
     if (trace && t == 0) trace[6] = stamp();
@@ -920,6 +950,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
   } else {
     // ================= warps 0-7: bias, (gather), epilogue, per tile
     if (t < bn) s_bias[t] = (p.bias != nullptr && nt0 * bn + t < p.N) ? __ldg(p.bias + nt0 * bn + t) : 0.f;
+    const EpiArgs ea = load_epi_args(p);
     pdl_wait();  // before reading this layer's activations (gather) or writing outputs
     const int quarter = warp & 3;
     const int half = warp >> 2;
@@ -1130,7 +1161,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
             }
           }
         }
-        if (row < valid_rows) epi16(p, sbias, ro, lb, m0, n0, bb, row, cb, v);
+        if (row < valid_rows) epi16(ea, sbias, ro, lb, m0, n0, bb, row, cb, v);
         if (more) tmem_ld_wait(r);
       }
       if (kPersistent) {  // this accumulator buffer may be overwritten by the MMA of tile it + 2

@@ -54,7 +54,7 @@ def child(model, scheme, batch=1):
     torch.cuda.synchronize()
     ctx = P.Context(0, P.config(**SCHEMES[scheme]))
     s = torch.cuda.current_stream().cuda_stream
-    time.sleep(0.05)
+    time.sleep(float(os.environ.get("PASK_COLD_SLEEP_MS", "50")) / 1e3)  # idle before the cold window
     torch.cuda.synchronize()
     t0 = time.perf_counter_ns()
     ctx.load_model(dm.graph, plan=False)

@@ -3,7 +3,7 @@
 # per-launch DRAM traffic per model, and full ncu captures of the contraction
 # and attention kernels.  Outputs in gpurun_out/ prefixed with $R (default r02).
 set -x
-R=${R:-r02}
+R=${R:-r03}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/${R}_build.log 2>&1
 python bench.py > gpurun_out/${R}_bench.json 2> gpurun_out/${R}_bench.err
@@ -26,3 +26,5 @@ ncu --set full --clock-control none --import-source on -k regex:pask_attention -
     -o gpurun_out/${R}_attention_full -f python bench.py --model bert_base_fa --steps 2 --warmup 1 --no-cpu-baseline \
     --cold-samples 0 > gpurun_out/${R}_ncu_full_attn.log 2>&1
 python -c "from paper_conf_dac_huangdxz25_b200 import build; build.build(force=True)" > /dev/null 2>&1
+python scripts/trace_inference.py resnet50 > gpurun_out/${R}_trace_resnet50.log 2>&1
+python scripts/trace_inference.py resnet50 --clock > gpurun_out/${R}_trace_clock_resnet50.log 2>&1
