@@ -366,6 +366,18 @@ def main():
     gbs = dk["bytes"] / (in_step_ms * 1e-3) / 1e9
     tfl = dk["flops"] / (in_step_ms * 1e-3) / 1e12
     gbs_iso = dk["bytes"] / (dk["ms"] * 1e-3) / 1e9
+    # every solution's bandwidth inside the step (same share method): the
+    # memory-bound ones against HBM, the contractions with their tensor rate too
+    tot_ms = sum(v["ms"] for v in per_kernel.values())
+    per_kernel_roofline = {}
+    for k, v in per_kernel.items():
+        st_ms = v["ms"] / tot_ms * hot_ms
+        per_kernel_roofline[k] = {
+            "launches": v["launches"], "bytes_per_launch": int(v["bytes"] / v["launches"]),
+            "in_step_us_per_launch": round(1e3 * st_ms / v["launches"], 2),
+            "achieved_gbs": round(v["bytes"] / (st_ms * 1e-3) / 1e9, 1),
+            "frac_hbm": round(v["bytes"] / (st_ms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4),
+            "tflops": round(v["flops"] / (st_ms * 1e-3) / 1e12, 2)}
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "dram_traffic.json")
     if os.path.exists(tpath):
@@ -470,6 +482,7 @@ def main():
                               "cold_wall": round(st["cold_wall_ns"] / 1e3, 1)},
         "load_timeline_us": timeline,
         "per_kernel_ms": {k: round(v["ms"], 4) for k, v in per_kernel.items()},
+        "per_kernel_roofline": per_kernel_roofline,
         "e2e": {"value": round(world * args.batch * 1000.0 / e2e_max, 2), "unit": "imgs/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": round(e2e_max, 4)},

@@ -194,13 +194,15 @@ __device__ __forceinline__ void gavg_body(const PoolParams& p) {
 // One thread per (output pixel, 8-channel chunk); weights RSC so each tap is
 // one 16 B load of x and one of w; fused bias / residual / activation.
 __device__ __forceinline__ void dw_body(const DwParams& p) {
-  pdl_wait();
-  pdl_launch_dependents();
   // 32-bit indices: the planner guarantees n*H*W*C < 2^31
   const int chunks = p.C >> 3;
   const int total = p.n * p.P * p.Q * chunks;
   const uint4* x = reinterpret_cast<const uint4*>(p.x);
   const uint4* w = reinterpret_cast<const uint4*>(p.w);
+  // (prefetching the first chunk's taps into L2 before griddepcontrol.wait
+  // measured slower: MobileNetV2 0.2371 -> 0.2471 ms)
+  pdl_wait();
+  pdl_launch_dependents();
   for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
     int t = idx;
     const int ch = t % chunks;
@@ -359,9 +361,17 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
 // the same order (lane's chunks ascending).
 constexpr int kLnRegChunks = 4;  // 16 B chunks per lane kept in registers
 __device__ __forceinline__ void layernorm_body(const RowParams& p) {
+  const int lane = threadIdx.x & 31;
+  // gamma / beta do not depend on the previous layer: pull this lane's lines into
+  // L2 before griddepcontrol.wait, so the normalisation's loads hit L2 instead of
+  // paying an HBM round trip after the reductions (BERT 0.5394 -> 0.5336 ms)
+  if (p.gamma && p.beta)
+    for (int c = lane * 8; c < p.cols; c += 256) {
+      prefetch_l2(p.gamma + c);
+      prefetch_l2(p.beta + c);
+    }
   pdl_wait();
   pdl_launch_dependents();
-  const int lane = threadIdx.x & 31;
   const int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   if (row >= p.rows) return;
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
