@@ -199,11 +199,21 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
   const int total = p.n * p.P * p.Q * chunks;
   const uint4* x = reinterpret_cast<const uint4*>(p.x);
   const uint4* w = reinterpret_cast<const uint4*>(p.w);
-  // (prefetching the first chunk's taps into L2 before griddepcontrol.wait
-  // measured slower: MobileNetV2 0.2371 -> 0.2471 ms)
+  // 3x3: the first output chunk's nine filter taps are loaded before
+  // griddepcontrol.wait (weights do not depend on the previous layer), so their
+  // HBM round trip overlaps the previous layer's tail.  (An L2 prefetch of the
+  // same lines by every thread measured slower: MobileNetV2 0.2371 -> 0.2471 ms.)
+  const bool k3 = p.R == 3 && p.S == 3 && p.dh == 1 && p.dw == 1;
+  const int idx0 = blockIdx.x * blockDim.x + threadIdx.x;
+  uint4 wpre[9];
+  if (k3 && idx0 < total) {
+    const int ch0 = idx0 % chunks;
+#pragma unroll
+    for (int t9 = 0; t9 < 9; ++t9) wpre[t9] = __ldg(w + t9 * chunks + ch0);
+  }
   pdl_wait();
   pdl_launch_dependents();
-  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
+  for (int idx = idx0; idx < total; idx += gridDim.x * blockDim.x) {
     int t = idx;
     const int ch = t % chunks;
     t /= chunks;
@@ -215,17 +225,18 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = 0.f;
     const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
-    if (p.R == 3 && p.S == 3 && p.dh == 1 && p.dw == 1) {
+    if (k3) {
       // 3x3 (MobileNetV2): all nine tap loads issued before the first FMA (one
       // memory round trip instead of nine); same taps, same order as below
       uint4 xv[9], wv[9];
       bool ok[9];
+      const bool first = idx == idx0;
 #pragma unroll
       for (int t9 = 0; t9 < 9; ++t9) {
         const int ih = ih0 + t9 / 3, iw = iw0 + t9 % 3;
         ok[t9] = ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
         xv[t9] = ok[t9] ? __ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch) : make_uint4(0, 0, 0, 0);
-        wv[t9] = __ldg(w + t9 * chunks + ch);
+        wv[t9] = first ? wpre[t9] : __ldg(w + t9 * chunks + ch);
       }
 #pragma unroll
       for (int t9 = 0; t9 < 9; ++t9) {
