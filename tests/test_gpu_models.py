@@ -234,3 +234,41 @@ def test_branches_bitwise(graph):
     for L in spec["layers"]:
         np.testing.assert_array_equal(got[L["out"]], dm2.read_raw(L["out"]))
     ctx2.close()
+
+
+_STORE_MODE_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+from tests.gpu_harness import run_model
+from workloads import build_model
+spec, x = build_model(sys.argv[2])
+dm, ctx, _ = run_model(spec, x)
+np.savez(sys.argv[3], **{L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]})  # bf16 -> f64 is exact
+ctx.close()
+"""
+
+
+@pytest.mark.parametrize("name", ["resnet50", "bert_base"])
+def test_direct_and_staged_epilogue_bitwise(name, tmp_path):
+    """The direct epilogue (c_tma = 2: 256-bit stores from registers, the default)
+    and the staged one (smem tile + TMA tensor store, PASK_STAGED_STORE=1) write
+    bitwise identical outputs for every layer: same arithmetic, only the store
+    path differs (DESIGN.md §6 K6 epilogue step 5).  Each mode runs in its own
+    process (the switch is read once per process)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    outs = {}
+    for mode in ("direct", "staged"):
+        env = dict(os.environ)
+        env.pop("PASK_STAGED_STORE", None)
+        if mode == "staged":
+            env["PASK_STAGED_STORE"] = "1"
+        path = str(tmp_path / f"{mode}.npz")
+        r = subprocess.run([sys.executable, "-c", _STORE_MODE_CHILD, root, name, path], env=env,
+                           capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-2000:]
+        outs[mode] = np.load(path)
+    for k in outs["direct"].files:
+        np.testing.assert_array_equal(outs["direct"][k], outs["staged"][k], err_msg=k)
