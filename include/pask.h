@@ -201,7 +201,12 @@ typedef struct {
                              CUfunction `pask_mem`, and conv_1x1 / gemm run on the generic
                              implicit-GEMM function -- one upload makes a whole family
                              resident; the plan (Algorithm 1) is unchanged, kernels_loaded
-                             counts the uploaded functions                                   */
+                             counts the uploaded functions; the families object is loaded
+                             in the smallest variant whose memory cases cover every
+                             solution the plan desires or binds (all / CNN / CNN +
+                             depthwise / transformer);
+                         3 = one CUfunction `pask_all` for both families (D10:
+                             one upload, measured slower on the hot path; not the default) */
   int32_t interleave; /* 0 = load-first (default): the first inference launches once every
                          planned kernel is uploaded -- on this driver a code upload waits for
                          all running GPU work, so
@@ -358,7 +363,8 @@ const char *pask_kernel_name(int32_t kernel_id);
  * code-object packaging `packaging` (pask_config.packaging): its own entry for
  * packaging 0 / 1; for packaging 2 the operator family's entry ("pask_mem" for
  * layout / dw / pool / gavg / softmax / LayerNorm, "pask_conv_igemm" for
- * igemm / conv_1x1 / gemm, D8).  "" for a bad id.  Host only. */
+ * igemm / conv_1x1 / gemm, D8); for packaging 3 "pask_all" for all of
+ * those (D10).  "" for a bad id.  Host only. */
 const char *pask_kernel_function(int32_t kernel_id, int32_t packaging);
 
 #ifdef __cplusplus
