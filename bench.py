@@ -333,6 +333,31 @@ def main():
             e2e_s.append(b - a)
     e2e_ms = 1e3 * statistics.mean(e2e_s)
 
+    # ---------------- hot through the direct-issue path (SURVEY.md §8(d) protocol:
+    # the paper's "Ideal", PAPER.md:178 -- the cold start's own issue path without
+    # any loading), L2 flushed like the timed loop; a separate context, graph off
+    if args.graph:
+        dctx = P.Context(local_rank, P.config(packaging=args.packaging, graph=0, branches=args.branches))
+        dctx.load_model(dm.graph, plan=False)
+        for _ in range(args.warmup):
+            flush()
+            dctx.infer(sp)
+        torch.cuda.synchronize()
+        dev_ = []
+        for i in range(args.steps):
+            if not args.no_flush:
+                flush()
+            a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a_.record(stream)
+            dctx.infer(sp)
+            b_.record(stream)
+            dev_.append((a_, b_))
+        torch.cuda.synchronize()
+        hot_direct_ms = statistics.mean(a_.elapsed_time(b_) for a_, b_ in dev_)
+        dctx.close()
+    else:
+        hot_direct_ms = hot_ms
+
     # ---------------- per-kernel roofline: instrumented pass (separate context)
     ictx = P.Context(local_rank, P.config(instrument=1))
     iplan = ictx.load_model(dm.graph)
@@ -400,7 +425,8 @@ def main():
                 "l2": "flushed before each inference (weights from HBM)"}
 
     # ---------------- max over ranks
-    hot_max, cold_max, e2e_max, warm_max = reduce_max([hot_ms, cold_ms, e2e_ms, hot_warm_ms], dist)
+    hot_max, cold_max, e2e_max, warm_max, direct_max = reduce_max(
+        [hot_ms, cold_ms, e2e_ms, hot_warm_ms, hot_direct_ms], dist)
     ctx.close()
     if rank != 0:
         if dist:
@@ -467,6 +493,10 @@ def main():
                                    "(scripts/cold_samples.py child, same model / packaging); "
                                    "cold_over_hot uses the median"},
         "hot_l2_warm_ms": round(warm_max, 4),
+        "hot_direct_ms": round(direct_max, 4),
+        "cold_over_hot_direct": round(cold_med / direct_max, 3),
+        "hot_direct_how": "direct cuLaunchKernelEx per layer (the cold start's issue path, no loading: the "
+                          "paper's Ideal, SURVEY.md §8(d)), L2 flushed, separate context",
         "kernels_loaded": st["kernels_loaded"],
         "kernels_loaded_names": loaded,
         "solutions_bound": solutions,
