@@ -239,13 +239,14 @@ def test_branches_issue_side_nodes_after_their_producer(name):
         assert sum(1 for _, kind in launches if kind == 3) == len(side)
 
 
-@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnn"), ("mobilenet_v2", "dw"),
+@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnn"), ("mobilenet_v2", "dwg"),
                                           ("bert_base", "tf"), ("bert_base_fa", "tf")])
 def test_family_variant_covers_the_plan(name, variant):
     """Packaging 2 (D8): the families object is loaded in the smallest
     variant whose memory-bound cases cover every solution the plan desires or
-    binds (CNN: layout / pool / global-average pool / softmax; + depthwise for
-    MobileNetV2; softmax / LayerNorm for BERT); one code object, whose bytes are
+    binds (CNN: layout / pool / global-average pool / softmax; layout /
+    depthwise / global-average pool / softmax for MobileNetV2; softmax /
+    LayerNorm for BERT); one code object, whose bytes are
     that variant's image (attention keeps its own object)."""
     from paper_conf_dac_huangdxz25_b200 import build as B
     spec, _ = build_model(name)
