@@ -155,6 +155,18 @@ def cores_used():
         return os.cpu_count()
 
 
+def cpu_model():
+    """The host CPU's model name (state the CPU the oracle ran on)."""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def run_reference(args, spec, x, rank):
     if rank != 0:
         return
@@ -169,7 +181,7 @@ def run_reference(args, spec, x, rank):
         "data": "synthetic", "config": {"workload": args.workload_name, "global_batch": 1,
                                         "model": args.model},
         "cpu_baseline": {"value": round(val, 4), "unit": "imgs/s", "cores": cores_used(),
-                         "kind": "oracle",
+                         "kind": "oracle", "cpu": cpu_model(),
                          "sample": f"{len(ts)} full fp64 numpy-oracle forwards of a batch-{args.batch} input"},
         "e2e": {"value": round(val, 4), "unit": "imgs/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
@@ -454,7 +466,7 @@ def main():
     if not args.no_cpu_baseline and world == 1:
         ts = time_oracle(spec, x, 5, 20.0)
         cpu = {"value": round(args.batch / statistics.mean(ts), 4), "unit": "imgs/s", "cores": cores_used(),
-               "kind": "oracle",
+               "kind": "oracle", "cpu": cpu_model(),
                "sample": f"{len(ts)} full fp64 numpy-oracle forwards of a batch-{args.batch} {args.model} input"}
 
     st = cold_stats
