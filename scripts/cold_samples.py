@@ -29,6 +29,7 @@ SCHEMES = {
     "pask_single_function": dict(packaging=3),        # both families in one CUfunction (D10)
     "pask_families_branches": dict(packaging=2, branches=1),  # bench default: + side stream (D9)
     "pask_families_branches_1s": dict(packaging=2, branches=1),  # ... cold issue on one stream
+    "pask_families_branches_noevw": dict(packaging=2, branches=1),  # ... events not warmed at create
     "pask_i": dict(reuse=0),                          # PaSK-I: proactive, no reuse
     "pask_r": dict(search=1),                         # PaSK-R: naive (exhaustive-order) search
     "reactive": dict(proactive=0, reuse=0),           # Baseline analog: lazy load at first launch
@@ -39,7 +40,8 @@ SCHEMES = {
     "pask_encfirst": dict(),                          # experiment: caller encodes, then uploads
 }
 SCHEME_ENV = {"pask_encfirst": {"PASK_ENCODE_FIRST": "1"},
-              "pask_families_branches_1s": {"PASK_DIRECT_ONE_STREAM": "1"}}
+              "pask_families_branches_1s": {"PASK_DIRECT_ONE_STREAM": "1"},
+              "pask_families_branches_noevw": {"PASK_NO_EVENT_WARM": "1"}}
 
 
 def child(model, scheme, batch=1):
