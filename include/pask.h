@@ -224,6 +224,15 @@ typedef struct {
                          main chain (D9); 0 = one stream, node order.  Ignored
                          with instrument = 1.  Same kernels and parameters either way:
                          outputs are bitwise identical                                       */
+  int32_t timeline;   /* 1 = every kernel stamps its first-CTA start / last-CTA end (%globaltimer)
+                         into a ctx-owned device buffer, so pask_sync can report the GPU busy
+                         time of an inference without events between the layers (PDL kept):
+                         gpu_busy_ns = union of the node intervals, the cold start's GPU
+                         utilisation of Fig. 6(b).  Two atomics per CTA   */
+  int32_t no_prefault; /* 1 = pask_create does not touch the host pages of the embedded code
+                         objects, so the first library parse inside the cold window also pays
+                         the page faults of reading the image (the Baseline's ELF read,
+                         PAPER.md:29); 0 (default) = prefault at create (D8)        */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;
@@ -250,7 +259,10 @@ typedef struct {
   uint64_t issue_ns;           /* time inside cuLaunchKernelEx calls             */
   uint64_t encode_ns;          /* CUtensorMap encoding + parameter packing        */
   uint64_t gpu_span_ns;        /* first launch -> last kernel end, last inference */
-  uint64_t gpu_busy_ns;        /* sum of per-kernel times (instrument = 1 only)   */
+  uint64_t gpu_busy_ns;        /* GPU busy time of the last synced inference: the
+                                  union of the kernels' [start, end] intervals
+                                  (timeline = 1), or the sum of per-kernel event
+                                  times (instrument = 1); 0 otherwise               */
   uint64_t cold_wall_ns;       /* pask_load_model entry -> first inference done   */
   uint64_t infer_count;
   uint64_t launches;           /* kernel launches issued so far                   */
@@ -260,21 +272,40 @@ typedef struct {
   uint64_t last_launch_ns;
   uint64_t encode_begin_ns;    /* launch-parameter encoding window, ns after      */
   uint64_t encode_end_ns;      /*   pask_load_model entry                         */
+  uint64_t kernel_span_ns;     /* timeline = 1: first kernel start -> last kernel end
+                                  (%globaltimer) of the last synced inference       */
+  uint64_t prefault_ns;        /* pask_create's host page touch of the code objects
+                                  (outside the cold window; 0 with no_prefault)     */
+  uint64_t prefault_bytes;
+  int32_t max_cluster;         /* largest split-K cluster this device can co-schedule
+                                  (cuOccupancyMaxActiveClusters; 16 or 8)           */
+  int32_t reserved0;
 } pask_stats_t;
 
 /* Library version (PASK_VERSION). */
 int pask_version(void);
 
-/* Create a context bound to the device's primary context (the one PyTorch
- * uses) and start the (idle) helper/loader thread.  Also touches the host pages
- * of the embedded code objects this packaging may load (host residency of the
- * library image, D8; nothing is uploaded to the GPU).  cfg may be
+/* Create a context for `device` and start the (idle) helper / loader thread --
+ * the "two extra host threads" PASK spawns for loading and issuing
+ * (PAPER.md:95, §III-A; :164, §III-D).  The ctx retains the device's primary
+ * context (the one PyTorch uses) and releases it in pask_destroy; if the
+ * calling thread has a current context on ANOTHER device (or a non-primary
+ * context) the call fails with PASK_EINVAL instead of binding the wrong one.
+ * The ctx makes its context current on the calling thread of every later entry
+ * point.  Outside the cold window it also touches the host pages of the
+ * embedded code objects this packaging may load (host residency of the library
+ * image, D8; cfg.no_prefault skips it; nothing is uploaded to the
+ * GPU) and, with cfg.timeline, allocates the 64 KB stamp buffer.  cfg may be
  * NULL for defaults {reuse 1, search 0, milestone 0, proactive 2, pdl 1,
- * instrument 0, packaging 0, interleave 0}. */
+ * instrument 0, packaging 0, interleave 0, graph 0, catalog 0, branches 0,
+ * timeline 0, no_prefault 0}.  Errors: PASK_ECUDA (driver missing / failing),
+ * PASK_EINVAL (null out-pointer, device mismatch). */
 int pask_create(pask_ctx **ctx, int device, const pask_config *cfg);
 
-/* Host-only planning (no GPU needed): validate g, extract problems p_i, apply
- * the static choice s*_i and Algorithm 1.  plan_out: caller-allocated
+/* Host-only planning (no GPU needed): the parse step P_i and
+ * Algorithm 1 EXECUTIONPLAN over the categorical cache (PAPER.md:105-141,
+ * §III-B/C): validate g, extract problems p_i, apply the static choice s*_i
+ * (the library's "find") and Algorithm 1.  plan_out: caller-allocated
  * [g->n_nodes]; stats_out (may be NULL) receives n_nodes, kernels_loaded
  * (planned), queries, hits, lookups, plan_ns.  Deterministic: a pure function
  * of (graph shapes, cfg). */
@@ -297,7 +328,10 @@ int pask_workspace_bytes(const pask_graph *g, uint64_t *bytes);
 int pask_load_model(pask_ctx *ctx, const pask_graph *g, pask_binding *plan_out);
 
 /* Issue one inference on cuda_stream (a CUstream / cudaStream_t; NULL = legacy
- * default stream).  inputs / outputs: device pointers, one per graph input /
+ * default stream): the issue step I_i of every layer, each launched "at the
+ * earliest feasible time right after the loading" of its solution
+ * (Fig. 5; the hot path afterwards is the paper's Ideal,
+ * PAPER.md:178).  inputs / outputs: device pointers, one per graph input /
  * output, or NULL to use the tensors' bound dptr; a pointer different from the
  * bound one rebinds that tensor (re-encoding the affected launch parameters).
  * Blocks only while a needed kernel is still loading; returns after the last
@@ -328,7 +362,11 @@ int pask_promote(pask_ctx *ctx, int32_t target_catalog, int32_t *promoted);
  * (gpu_span_ns; cold_wall_ns after the first inference). */
 int pask_sync(pask_ctx *ctx);
 
-/* Copy the statistics (host only; call pask_sync first for GPU times). */
+/* Copy the statistics (host only; call pask_sync first for GPU times): the
+ * quantities of the paper's cold-start breakdown -- code loading, issue, GPU
+ * execution (Fig. 1(b); Fig. 7, :212-216), GPU busy for the
+ * utilisation of Fig. 6(b) (:208, :214) and the cache statistics of Fig. 9
+ * (queries, hits, lookups; :226-234).  Errors: PASK_EINVAL on null arguments. */
 int pask_stats(const pask_ctx *ctx, pask_stats_t *out);
 
 /* Cross-check with the driver: *state = 1 if kernel_id's CUfunction is loaded
@@ -349,6 +387,12 @@ int pask_kernel_timeline(const pask_ctx *ctx, int32_t kernel_id, uint64_t *load_
  * cfg.instrument = 1 (call pask_sync first).  ns_out: caller array of
  * n_nodes entries; PASK_ESTATE if the context is not instrumented. */
 int pask_node_times(const pask_ctx *ctx, uint64_t *ns_out, int32_t n_nodes);
+
+/* Per-node GPU intervals of the last synced inference of a timeline = 1 ctx:
+ * start_ns[i] / end_ns[i] = node i's first CTA start / last CTA end, ns after
+ * the inference's first kernel start (%globaltimer, ~0.25 us resolution); a
+ * node that did not run reports 0 / 0.  PASK_ESTATE without timeline. */
+int pask_node_intervals(const pask_ctx *ctx, uint64_t *start_ns, uint64_t *end_ns, int32_t n_nodes);
 
 /* Join the loader thread, unload the library and free host state. */
 int pask_destroy(pask_ctx *ctx);

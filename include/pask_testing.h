@@ -12,7 +12,9 @@
  *   - cuLaunchKernelEx records the launched kernel id (the catalog id whose
  *     code object was loaded) and whether that kernel had been loaded before
  *     the launch;
- *   - stream capture is unsupported (CUDA_ERROR_NOT_SUPPORTED).
+ *   - stream capture logs the captured launches; a graph replay launches nothing;
+ *   - device memory (only the timeline buffer) is host memory;
+ *   - it is compiled only into libpask_testing.so, never into libpask.so.
  */
 #ifndef PASK_TESTING_H
 #define PASK_TESTING_H
@@ -36,6 +38,18 @@ int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail_kernel);
  * the contraction family as PASK_K_CONV_IGEMM.  Returns the number of events
  * (writes at most cap). */
 int32_t pask_test_fake_log(int32_t *out, int32_t *kinds, int32_t cap);
+
+/* Knobs of the fake driver (reset by pask_test_fake_driver):
+ *   PASK_FAKE_OCCUPANCY            set what cuOccupancyMaxActiveClusters reports
+ *                                  for a 16-CTA cluster (default 1; 0 = cannot
+ *                                  co-schedule one); returns 0
+ *   PASK_FAKE_CURRENT_DEVICE       make device `value`'s primary context current
+ *                                  (default 0); returns 0
+ *   PASK_FAKE_MAX_CLUSTER_LAUNCHED returns the largest cluster size (z) launched
+ *                                  since the last reset; value ignored
+ * Unknown knob: -1. */
+enum { PASK_FAKE_OCCUPANCY = 1, PASK_FAKE_CURRENT_DEVICE = 2, PASK_FAKE_MAX_CLUSTER_LAUNCHED = 3 };
+int32_t pask_test_fake_knob(int32_t knob, int32_t value);
 
 #ifdef __cplusplus
 }

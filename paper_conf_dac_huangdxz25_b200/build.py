@@ -22,9 +22,13 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 KERNEL_SRC = [os.path.join(CSRC, "kernels", f) for f in
               ("pask_kernels.cu", "conv_gemm.cuh", "attention.cuh", "elementwise.cuh", "ptx.cuh",
                "pask_params.h")]
-HOST_SRC = [os.path.join(CSRC, "runtime", f) for f in ("pask.cpp", "plan.cpp", "driver.cpp", "fake_driver.cpp")]
-HOST_DEPS = HOST_SRC + [os.path.join(CSRC, "runtime", f) for f in
-                         ("plan.h", "driver.h", "exports.map")] + [
+HOST_SRC = [os.path.join(CSRC, "runtime", f) for f in ("pask.cpp", "plan.cpp", "driver.cpp")]
+# the fake CUDA driver (include/pask_testing.h) is compiled only into the
+# test-only library libpask_testing.so, never into the product libpask.so
+TEST_SRC = [os.path.join(CSRC, "runtime", "fake_driver.cpp")]
+TEST_LIB = os.path.join(PKG, "libpask_testing.so")
+HOST_DEPS = HOST_SRC + TEST_SRC + [os.path.join(CSRC, "runtime", f) for f in
+                                   ("plan.h", "driver.h", "tuning.h", "exports.map")] + [
     os.path.join(CSRC, "kernels", "pask_params.h"),
     os.path.join(os.path.dirname(PKG), "include", "pask.h"),
     os.path.join(os.path.dirname(PKG), "include", "pask_testing.h")]
@@ -57,8 +61,10 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # LayerNorm 5); the runtime loads the smallest covering the model's solutions
 # (dwg = depthwise + global pool without the windowed pool: MobileNetV2).
 # Packaging 3 (D10): both families behind the single entry `pask_all`.
-FAMILY_VARIANTS = {"pask_families": 0x3f, "pask_families_cnn": 0x1d, "pask_families_dw": 0x1f,
-                   "pask_families_dwg": 0x1b, "pask_families_tf": 0x30}
+# Smallest first: the runtime takes the first variant covering the plan (the
+# table is generated into _build/spec_catalog.h as PASK_FAMILY_VARIANTS).
+FAMILY_VARIANTS = {"pask_families_tf": 0x30, "pask_families_dwg": 0x1b, "pask_families_cnn": 0x1d,
+                   "pask_families_dw": 0x1f, "pask_families": 0x3f}
 EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"]}
 EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}"] for k, m in FAMILY_VARIANTS.items()}
 
@@ -90,7 +96,7 @@ def _gen_spec_sources():
         n = spec_name(sp)
         ker.append(f"#if !defined(PASK_NO_SPECS) && (!defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_{n})\n"
                    f"__global__ void __launch_bounds__(kGemmThreads, 1) {n}(const __grid_constant__ GemmParams p) "
-                   f"{{ conv_gemm_body<true, FixGeo<{', '.join(map(str, sp))}>>(p); }}\n#endif\n")
+                   f"{{ TimelineScope ts(p.tl); conv_gemm_body<true, FixGeo<{', '.join(map(str, sp))}>>(p); }}\n#endif\n")
     host = ["// generated by build.py: the specialised conv solutions (catalog ids PASK_NUM_KERNELS + i)",
             "#pragma once", "namespace pask {",
             "struct SpecEntry { int r, s, st, pd, dl, c; const char* name; };",
@@ -99,12 +105,29 @@ def _gen_spec_sources():
     host += ["    {%d, %d, %d, %d, %d, %d, \"%s\"}," % (*sp, spec_name(sp)) for sp in SPECS]
     host += ["};", "}  // namespace pask", ""]
     host += ["#define PASK_SPEC_IMAGES(X) \\"] + [f"  X({spec_name(sp)}) \\" for sp in SPECS] + [""]
+    host += ["// packaging 2 families variants (name, memory-case mask), smallest first",
+             "#define PASK_FAMILY_VARIANTS(X) \\"] + \
+        [f"  X({k}, {m:#x}) \\" for k, m in FAMILY_VARIANTS.items()] + [""]
     for path, text in ((os.path.join(BUILD, "spec_kernels.inc"), "".join(ker)),
                        (os.path.join(BUILD, "spec_catalog.h"), "\n".join(host))):
         old = open(path).read() if os.path.exists(path) else None
         if old != text:
             with open(path, "w") as f:
                 f.write(text)
+
+
+def _defines_stamp():
+    """_build/defines.stamp: rewritten only when the build-affecting environment
+    changes, so an experiment build (PASK_NVCC_DEFINES / PASK_LINEINFO) never
+    leaves stale fatbins behind."""
+    text = f"PASK_NVCC_DEFINES={os.environ.get('PASK_NVCC_DEFINES', '')}\n" \
+           f"PASK_LINEINFO={os.environ.get('PASK_LINEINFO', '')}\n"
+    path = os.path.join(BUILD, "defines.stamp")
+    old = open(path).read() if os.path.exists(path) else None
+    if old != text:
+        with open(path, "w") as f:
+            f.write(text)
+    return path
 
 
 def _nvcc_fatbin_cmd(out, defines=()):
@@ -153,7 +176,7 @@ def _build_locked(force: bool, verbose: bool) -> str:
     fatbin = os.path.join(BUILD, "pask.fatbin")
     names = KERNELS + list(EXTRA_OBJECTS) + [spec_name(sp) for sp in SPECS]
     per_kernel = [os.path.join(BUILD, k + ".fatbin") for k in names]
-    deps = KERNEL_SRC + [os.path.join(BUILD, "spec_kernels.inc")]
+    deps = KERNEL_SRC + [os.path.join(BUILD, "spec_kernels.inc"), os.path.abspath(__file__), _defines_stamp()]
     if force or any(_stale(f, deps) for f in [fatbin] + per_kernel):
         # the generic catalog as one code object, and one code object per kernel
         cmds = [(fatbin, _nvcc_fatbin_cmd(fatbin, ["-DPASK_NO_SPECS"]))]
@@ -177,22 +200,25 @@ def _build_locked(force: bool, verbose: bool) -> str:
                      f"{sym}_start:\n        .incbin \"{path}\"\n        .globl {sym}_end\n"
                      f"        .hidden {sym}_end\n{sym}_end:\n        .byte 0\n")
         fh.write('        .section .note.GNU-stack,"",@progbits\n')
-    if force or _stale(LIB, HOST_DEPS + [fatbin] + per_kernel + [os.path.join(BUILD, "spec_catalog.h")]):
+    host_deps = HOST_DEPS + [fatbin] + per_kernel + [os.path.join(BUILD, "spec_catalog.h"), _defines_stamp(),
+                                                      os.path.abspath(__file__)]
+    if force or _stale(LIB, host_deps) or _stale(TEST_LIB, host_deps):
         cxx = os.environ.get("CXX", "g++")
         flags = ["-O2", "-std=c++17", "-fPIC", "-fvisibility=hidden", "-Wall", "-Wno-unused-function",
                  f"-I{CUDA}/include", f"-I{BUILD}"]
         flags += os.environ.get("PASK_NVCC_DEFINES", "").split()  # experiment builds: same -D for host
-        objs = []
-        for src in HOST_SRC:
+        objs = {}
+        for src in HOST_SRC + TEST_SRC:
             obj = os.path.join(BUILD, os.path.basename(src) + ".o")
             _run([cxx, *flags, "-c", src, "-o", obj])
-            objs.append(obj)
+            objs[src] = obj
         fobj = os.path.join(BUILD, "fatbin.o")
         _run([cxx, "-c", asm, "-o", fobj])
-        tmp = LIB + ".tmp"
-        _run([cxx, "-shared", "-o", tmp, *objs, fobj, "-ldl", "-lpthread", "-Wl,--no-undefined",
-              "-Wl,--version-script=" + os.path.join(CSRC, "runtime", "exports.map")])
-        shutil.move(tmp, LIB)
+        for lib, srcs in ((LIB, HOST_SRC), (TEST_LIB, HOST_SRC + TEST_SRC)):
+            tmp = lib + ".tmp"
+            _run([cxx, "-shared", "-o", tmp, *[objs[x] for x in srcs], fobj, "-ldl", "-lpthread",
+                  "-Wl,--no-undefined", "-Wl,--version-script=" + os.path.join(CSRC, "runtime", "exports.map")])
+            shutil.move(tmp, lib)
     return LIB
 
 

@@ -9,6 +9,8 @@
 
 using namespace pask;
 
+static_assert(kTimelineStride == 4096, "TimelineScope (ptx.cuh) hard-codes the end-slot offset");
+
 // PASK_MEM_MASK (bit per MemKind) selects the memory-family cases compiled into
 // a code object: packaging 2 ships the families object in variants (all cases,
 // CNN, CNN + depthwise, transformer) and loads the smallest one covering the
@@ -25,12 +27,12 @@ using namespace pask;
 // The memory-bound family: the solution's own body selected by p.kind.
 __device__ __forceinline__ void mem_dispatch(const MemParams& p) {
   switch (p.kind) {
-    PASK_MEM_CASE(MEM_LAYOUT, layout_body(p.l))
-    PASK_MEM_CASE(MEM_DW, dw_body(p.d))
-    PASK_MEM_CASE(MEM_POOL, pool_body(p.p))
-    PASK_MEM_CASE(MEM_GAVG, gavg_body(p.p))
-    PASK_MEM_CASE(MEM_SOFTMAX, softmax_body(p.r))
-    PASK_MEM_CASE(MEM_LAYERNORM, layernorm_body(p.r))
+    PASK_MEM_CASE(MEM_LAYOUT, TimelineScope ts(p.l.tl); layout_body(p.l))
+    PASK_MEM_CASE(MEM_DW, TimelineScope ts(p.d.tl); dw_body(p.d))
+    PASK_MEM_CASE(MEM_POOL, TimelineScope ts(p.p.tl); pool_body(p.p))
+    PASK_MEM_CASE(MEM_GAVG, TimelineScope ts(p.p.tl); gavg_body(p.p))
+    PASK_MEM_CASE(MEM_SOFTMAX, TimelineScope ts(p.r.tl); softmax_body(p.r))
+    PASK_MEM_CASE(MEM_LAYERNORM, TimelineScope ts(p.r.tl); layernorm_body(p.r))
     default: __trap();
   }
 }
@@ -40,6 +42,7 @@ extern "C" {
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_layout
 // PASK_K_LAYOUT
 __global__ void __launch_bounds__(256) pask_layout(const __grid_constant__ LayoutParams p) {
+  TimelineScope ts(p.tl);
   layout_body(p);
 }
 #endif
@@ -47,6 +50,7 @@ __global__ void __launch_bounds__(256) pask_layout(const __grid_constant__ Layou
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_conv_igemm
 // PASK_K_CONV_IGEMM: generic implicit-GEMM conv (A by gather, or TMA for 1x1 s1 p0)
 __global__ void __launch_bounds__(kGemmThreads, 1) pask_conv_igemm(const __grid_constant__ GemmParams p) {
+  TimelineScope ts(p.tl);
   conv_gemm_body<true>(p);
 }
 #endif
@@ -55,6 +59,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1) pask_conv_igemm(const __grid_
 // PASK_K_CONV_IGEMM_PT: the implicit-GEMM conv as persistent tiles (<= #SMs CTAs
 // loop over the tiles, double-buffered TMEM accumulator / staging, store agent)
 __global__ void __launch_bounds__(kGemmThreadsPT, 1) pask_conv_igemm_pt(const __grid_constant__ GemmParams p) {
+  TimelineScope ts(p.tl);
   conv_gemm_body_pt<true>(p);
 }
 #endif
@@ -62,28 +67,39 @@ __global__ void __launch_bounds__(kGemmThreadsPT, 1) pask_conv_igemm_pt(const __
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_conv_1x1
 // PASK_K_CONV_1X1: specialised 1x1 / stride 1 / pad 0 conv (A by TMA only)
 __global__ void __launch_bounds__(kGemmThreads, 1) pask_conv_1x1(const __grid_constant__ GemmParams p) {
+  TimelineScope ts(p.tl);
   conv_gemm_body<false>(p);
 }
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_conv_dw
 // PASK_K_CONV_DW
-__global__ void __launch_bounds__(256) pask_conv_dw(const __grid_constant__ DwParams p) { dw_body(p); }
+__global__ void __launch_bounds__(256) pask_conv_dw(const __grid_constant__ DwParams p) {
+  TimelineScope ts(p.tl);
+  dw_body(p);
+}
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_pool
 // PASK_K_POOL
-__global__ void __launch_bounds__(256) pask_pool(const __grid_constant__ PoolParams p) { pool_body(p); }
+__global__ void __launch_bounds__(256) pask_pool(const __grid_constant__ PoolParams p) {
+  TimelineScope ts(p.tl);
+  pool_body(p);
+}
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_pool_gavg
 // PASK_K_POOL_GAVG
-__global__ void __launch_bounds__(128) pask_pool_gavg(const __grid_constant__ PoolParams p) { gavg_body(p); }
+__global__ void __launch_bounds__(128) pask_pool_gavg(const __grid_constant__ PoolParams p) {
+  TimelineScope ts(p.tl);
+  gavg_body(p);
+}
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_gemm
 // PASK_K_GEMM: batched GEMM (A K-major by TMA; B K- or MN-major by TMA)
 __global__ void __launch_bounds__(kGemmThreads, 1) pask_gemm(const __grid_constant__ GemmParams p) {
+  TimelineScope ts(p.tl);
   conv_gemm_body<false>(p);
 }
 #endif
@@ -91,18 +107,25 @@ __global__ void __launch_bounds__(kGemmThreads, 1) pask_gemm(const __grid_consta
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_attention
 // PASK_K_ATTENTION: fused QK^T -> softmax -> PV (tcgen05, scores in TMEM)
 __global__ void __launch_bounds__(192, 1) pask_attention(const __grid_constant__ AttnParams p) {
+  TimelineScope ts(p.tl);
   attention_body(p);
 }
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_softmax
 // PASK_K_SOFTMAX
-__global__ void __launch_bounds__(256) pask_softmax(const __grid_constant__ RowParams p) { softmax_body(p); }
+__global__ void __launch_bounds__(256) pask_softmax(const __grid_constant__ RowParams p) {
+  TimelineScope ts(p.tl);
+  softmax_body(p);
+}
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_layernorm
 // PASK_K_LAYERNORM
-__global__ void __launch_bounds__(256) pask_layernorm(const __grid_constant__ RowParams p) { layernorm_body(p); }
+__global__ void __launch_bounds__(256) pask_layernorm(const __grid_constant__ RowParams p) {
+  TimelineScope ts(p.tl);
+  layernorm_body(p);
+}
 #endif
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_mem
@@ -119,10 +142,12 @@ __global__ void __launch_bounds__(256) pask_mem(const __grid_constant__ MemParam
 // upload for a whole CNN / transformer catalog.  Same bodies as the solutions' own
 // entries, so outputs are bitwise equal.
 __global__ void __launch_bounds__(kGemmThreads, 1) pask_all(const __grid_constant__ AllParams p) {
-  if (p.g.family == 0)
+  if (p.g.family == 0) {
+    TimelineScope ts(p.g.tl);
     conv_gemm_body<true>(p.g);
-  else
+  } else {
     mem_dispatch(p.m);
+  }
 }
 #endif
 

@@ -27,6 +27,13 @@ constexpr int kEpiWarpsPT = 8;
 constexpr int kEpiThreadsPT = 32 * kEpiWarpsPT;
 constexpr int kGemmThreadsPT = kEpiThreadsPT + 96;
 
+// pask_config.timeline (GPU busy during the cold start, Fig. 6(b)): node i's
+// kernel atomically lowers tl[i] to its first CTA's start and raises
+// tl[i + kTimelineStride] to its last CTA's end (%globaltimer ns).  The buffer
+// (2 x kTimelineStride u64) is owned by the ctx; graphs longer than
+// kTimelineStride nodes run without stamps.
+constexpr int kTimelineStride = 4096;
+
 // A-operand source of the contraction kernel.
 enum AMode : int32_t {
   A_TMA = 0,     // A is a plain K-major matrix: TMA tiled load (GEMM, 1x1 s1 p0 conv)
@@ -49,6 +56,7 @@ struct alignas(64) GemmParams {
   int32_t persistent;   // 1: grid of <= #SMs CTAs loops over the tiles, TMEM double-buffered
   int32_t n_tiles_total;  // m_tiles * n_tiles * batch (persistent)
   unsigned long long* trace;  // debug: per-CTA phase stamps (null in production)
+  unsigned long long* tl;     // pask_config.timeline: this node's [start, end] slots (null = off)
   int64_t ldc, off_c, stride_c;
   int32_t M, N, K, batch;
   int32_t num_kb;        // ceil(K / 64)
@@ -80,6 +88,7 @@ struct alignas(16) LayoutParams {
   const float* x;  // NCHW fp32
   void* y;         // NHWC bf16, c_out channels (c_out % 8 == 0)
   int32_t n, c, h, w, c_out;
+  unsigned long long* tl;  // pask_config.timeline slots (null = off)
 };
 
 struct alignas(16) PoolParams {
@@ -89,6 +98,7 @@ struct alignas(16) PoolParams {
   int32_t mode;   // 0 max, 1 avg
   int32_t count_include_pad;
   int32_t per_warp;  // 1: one warp per output chunk, lanes split the window (large windows)
+  unsigned long long* tl;  // pask_config.timeline slots (null = off)
 };
 
 struct alignas(16) DwParams {
@@ -99,6 +109,7 @@ struct alignas(16) DwParams {
   void* y;             // NHWC bf16 [n][P][Q][C]
   int32_t n, H, W, C, P, Q, R, S, sh, sw, ph, pw, dh, dw;
   int32_t act;
+  unsigned long long* tl;  // pask_config.timeline slots (null = off)
 };
 
 // Fused attention (PASK_K_ATTENTION): one CTA per (128-query tile, head, sequence).
@@ -112,6 +123,7 @@ struct alignas(64) AttnParams {
   uint32_t idesc_pv;     // M=128, N=64, A K-major, B MN-major
   uint32_t tmem_cols;    // power of two >= s_pad + 64
   uint32_t smem_bytes;
+  unsigned long long* tl;  // pask_config.timeline slots (null = off)
 };
 
 struct alignas(16) RowParams {
@@ -122,6 +134,7 @@ struct alignas(16) RowParams {
   int32_t rows, cols;
   float scale;  // softmax
   float eps;    // layernorm
+  unsigned long long* tl;  // pask_config.timeline slots (null = off)
 };
 
 // Operator-family entry (pask_config.packaging = 2): the memory-bound solutions

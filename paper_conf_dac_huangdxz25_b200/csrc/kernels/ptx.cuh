@@ -18,6 +18,20 @@ __device__ __forceinline__ unsigned long long globaltimer() {
   return t;
 }
 
+// pask_config.timeline: the kernel's [first CTA start, last CTA end] in
+// %globaltimer ns (start slot tl[0], end slot tl[kTimelineStride]).  Thread 0 of
+// each CTA stamps on entry and when it leaves the body; two relaxed 64-bit
+// atomics per CTA, none when tl is null (the default).
+struct TimelineScope {
+  unsigned long long* tl;
+  __device__ __forceinline__ explicit TimelineScope(unsigned long long* p) : tl(p) {
+    if (tl != nullptr && threadIdx.x == 0) atomicMin(tl, globaltimer());
+  }
+  __device__ __forceinline__ ~TimelineScope() {
+    if (tl != nullptr && threadIdx.x == 0) atomicMax(tl + 4096, globaltimer());
+  }
+};
+
 // ---------------------------------------------------------------- PDL
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_launch_dependents() {

@@ -70,6 +70,12 @@ void resolve() {
   PASK_RESOLVE(cuGraphLaunch)
   PASK_RESOLVE(cuGraphDestroy)
   PASK_RESOLVE(cuGraphExecDestroy)
+  PASK_RESOLVE(cuCtxGetDevice)
+  PASK_RESOLVE(cuOccupancyMaxActiveClusters)
+  PASK_RESOLVE(cuMemAlloc)
+  PASK_RESOLVE(cuMemFree)
+  PASK_RESOLVE(cuMemsetD8)
+  PASK_RESOLVE(cuMemcpyDtoH)
 #undef PASK_RESOLVE
   if (!all) {
     g_why = "a required CUDA driver entry point could not be resolved (driver too old?)";

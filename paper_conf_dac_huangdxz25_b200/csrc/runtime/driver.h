@@ -44,6 +44,12 @@ struct Driver {
   PASK_DRV_FN(cuGraphLaunch)
   PASK_DRV_FN(cuGraphDestroy)
   PASK_DRV_FN(cuGraphExecDestroy)
+  PASK_DRV_FN(cuCtxGetDevice)
+  PASK_DRV_FN(cuOccupancyMaxActiveClusters)
+  PASK_DRV_FN(cuMemAlloc)
+  PASK_DRV_FN(cuMemFree)
+  PASK_DRV_FN(cuMemsetD8)
+  PASK_DRV_FN(cuMemcpyDtoH)
 #undef PASK_DRV_FN
   bool ok = false;
 };

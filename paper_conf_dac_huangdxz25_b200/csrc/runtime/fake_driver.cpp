@@ -2,8 +2,10 @@
 // issuer host logic without a GPU.  Handles are small integers disguised as
 // pointers; a CUfunction encodes its catalog kernel id (found from the name).
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
+#include <algorithm>
 #include <chrono>
 #include <atomic>
 #include <mutex>
@@ -57,11 +59,51 @@ CUresult f_dev_get(CUdevice* d, int o) {
   *d = o;
   return CUDA_SUCCESS;
 }
+// contexts: device d's primary context is 0x10 + d; "current" is process-wide
+// here (device 0's primary by default, as after torch.cuda.set_device(0))
+std::atomic<uintptr_t> g_current{0x10};
+std::atomic<int32_t> g_occupancy{1};      // cuOccupancyMaxActiveClusters result
+std::atomic<int32_t> g_max_cluster_z{0};  // largest cluster launched
 CUresult f_ctx_get(CUcontext* c) {
-  *c = fake_handle<CUcontext>(0x10);
+  *c = fake_handle<CUcontext>(g_current.load());
   return CUDA_SUCCESS;
 }
-CUresult f_ctx_set(CUcontext) { return CUDA_SUCCESS; }
+CUresult f_ctx_set(CUcontext c) {
+  g_current.store(reinterpret_cast<uintptr_t>(c));
+  return CUDA_SUCCESS;
+}
+CUresult f_primary_retain(CUcontext* c, CUdevice d) {
+  *c = fake_handle<CUcontext>(0x10 + static_cast<uintptr_t>(d));
+  return CUDA_SUCCESS;
+}
+CUresult f_primary_release(CUdevice) { return CUDA_SUCCESS; }
+CUresult f_ctx_get_device(CUdevice* d) {
+  *d = static_cast<CUdevice>(g_current.load() - 0x10);
+  return CUDA_SUCCESS;
+}
+CUresult f_occupancy_clusters(int* n, CUfunction, const CUlaunchConfig*) {
+  *n = g_occupancy.load();
+  return CUDA_SUCCESS;
+}
+// device memory of the fake: host memory (only the timeline buffer uses it)
+CUresult f_mem_alloc(CUdeviceptr* p, size_t bytes) {
+  void* h = calloc(1, bytes);
+  if (!h) return CUDA_ERROR_OUT_OF_MEMORY;
+  *p = reinterpret_cast<CUdeviceptr>(h);
+  return CUDA_SUCCESS;
+}
+CUresult f_mem_free(CUdeviceptr p) {
+  free(reinterpret_cast<void*>(p));
+  return CUDA_SUCCESS;
+}
+CUresult f_memset_d8(CUdeviceptr p, unsigned char v, size_t n) {
+  memset(reinterpret_cast<void*>(p), v, n);
+  return CUDA_SUCCESS;
+}
+CUresult f_memcpy_dtoh(void* dst, CUdeviceptr src, size_t n) {
+  memcpy(dst, reinterpret_cast<const void*>(src), n);
+  return CUDA_SUCCESS;
+}
 CUresult f_lib_load(CUlibrary* lib, const void*, CUjit_option*, void**, unsigned int, CUlibraryOption*, void**,
                     unsigned int) {
   sleep_us(g_load_us);
@@ -110,6 +152,9 @@ CUresult f_launch(const CUlaunchConfig* cfg, CUfunction f, void**, void**) {
   }
   // 1: launch on the caller's stream, 3: on another stream (the branches side
   // stream, D9), 2: kernel not loaded (must never happen)
+  for (unsigned a = 0; a < cfg->numAttrs; ++a)
+    if (cfg->attrs[a].id == CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION)
+      g_max_cluster_z.store(std::max<int32_t>(g_max_cluster_z.load(), cfg->attrs[a].value.clusterDim.z));
   const uintptr_t sh = reinterpret_cast<uintptr_t>(cfg->hStream);
   const bool main_stream = sh == 0 || sh == g_capture_stream.load();
   log_event(id, !loaded ? 2 : (main_stream ? 1 : 3));
@@ -176,6 +221,14 @@ Driver make_fake() {
   d.cuDeviceGet = f_dev_get;
   d.cuCtxGetCurrent = f_ctx_get;
   d.cuCtxSetCurrent = f_ctx_set;
+  d.cuDevicePrimaryCtxRetain = f_primary_retain;
+  d.cuDevicePrimaryCtxRelease = f_primary_release;
+  d.cuCtxGetDevice = f_ctx_get_device;
+  d.cuOccupancyMaxActiveClusters = f_occupancy_clusters;
+  d.cuMemAlloc = f_mem_alloc;
+  d.cuMemFree = f_mem_free;
+  d.cuMemsetD8 = f_memset_d8;
+  d.cuMemcpyDtoH = f_memcpy_dtoh;
   d.cuLibraryLoadData = f_lib_load;
   d.cuLibraryUnload = f_lib_unload;
   d.cuLibraryGetKernel = f_lib_get_kernel;
@@ -221,6 +274,9 @@ PASK_API int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail
   memset(g_loaded, 0, sizeof(g_loaded));
   g_next_stream.store(0x40);
   g_capture_stream.store(0);
+  g_current.store(0x10);
+  g_occupancy.store(1);
+  g_max_cluster_z.store(0);
   if (enable) {
     g_fake = make_fake();
     driver_override(&g_fake);
@@ -228,6 +284,16 @@ PASK_API int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail
     driver_override(nullptr);
   }
   return 0;
+}
+
+PASK_API int32_t pask_test_fake_knob(int32_t knob, int32_t value) {
+  using namespace pask;
+  switch (knob) {
+    case PASK_FAKE_OCCUPANCY: g_occupancy.store(value); return 0;
+    case PASK_FAKE_CURRENT_DEVICE: g_current.store(0x10 + static_cast<uintptr_t>(value)); return 0;
+    case PASK_FAKE_MAX_CLUSTER_LAUNCHED: return g_max_cluster_z.load();
+    default: return -1;
+  }
 }
 
 PASK_API int32_t pask_test_fake_log(int32_t* out, int32_t* kinds, int32_t cap) {

@@ -65,8 +65,9 @@ struct GemmTiling {
 // Dynamic shared memory the contraction kernels may request (attribute set at load).
 constexpr uint32_t kMaxDynSmem = 220u * 1024u;
 // c_tma: output / residual go through smem staging + TMA (changes the smem size)
+// max_cluster: largest split-K cluster the device co-schedules (16 on a full B200)
 GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma,
-                       int32_t persistent_kernel = 0);
+                       int32_t persistent_kernel = 0, int32_t max_cluster = 16);
 // s* rule: a dense conv with more output rows than 148 SMs x 128-row tiles takes
 // the persistent-tile solution (PASK_K_CONV_IGEMM_PT)
 constexpr int64_t kPersistentRows = 148 * 128;

@@ -1,0 +1,45 @@
+// Tiling and issue constants of the runtime, and the experiment switches used
+// to measure the alternatives DESIGN.md reports.
+//
+// Release builds use the constants below.  A build with -DPASK_EXPERIMENTS
+// (PASK_NVCC_DEFINES="-DPASK_EXPERIMENTS" python -m paper_conf_dac_huangdxz25_b200.build)
+// also reads the PASK_* environment variables, ONCE (the first call of tuning(),
+// from pask_create / pask_plan on the caller's thread), and clamps every value
+// to the range the kernels support -- e.g. splits <= min(16, num_kb) is kept by
+// gemm_tiling regardless of PASK_SPLIT_MAX, and the device trace pointer is
+// only honoured in experiment builds.
+#pragma once
+#include <stdint.h>
+
+namespace pask {
+
+struct Tuning {
+  // gemm_tiling (plan.cpp)
+  int tile_target = 74;   // halve the N tile while the grid has fewer tiles than this
+  int bn_min = 64;        // ... but not below this N tile
+  int split_min_kb = 8;   // k-blocks each split-K slice keeps at least
+  int split_max = 8;      // largest portable split-K cluster
+  int split_fill = 2;     // tiles * splits * fill <= #SMs
+  int bn32_tiles = 8;     // unsplittable layers with <= this many tiles take 32-wide N tiles
+  // lowering (pask.cpp)
+  int gather_lag = 2;     // A_GATHER: k-blocks of cp.async in flight before publishing a slot
+  int pre_b = 0;          // weight k-blocks fetched before griddepcontrol.wait (0 = whole ring)
+  bool staged_store = false;  // stage every epilogue tile for a TMA store (c_tma = 1)
+  bool no_a64 = false;        // never use 64-row A boxes
+  bool no_im2col = false;     // A_GATHER instead of TMA im2col
+  // issue / loading (pask.cpp)
+  bool encode_first = false;       // proactive 2: encode, then upload (instead of concurrently)
+  bool debug_cold = false;         // print per-launch host times of the cold inference
+  bool fork_no_pdl = false;        // branches: drop PDL after a fork record
+  bool join_no_pdl = false;        // branches: drop PDL after a join wait
+  bool direct_one_stream = false;  // branches: direct issue on one stream
+  bool no_event_warm = false;      // pask_create: do not pre-record the timing events
+  // device phase trace (experiment builds only)
+  int trace_node = -2;             // node index, -1 = all, -2 = off
+  uint64_t trace_ptr = 0;          // device address of the trace buffer
+  bool trace_clock = false;        // SM clock64 cycles instead of %globaltimer
+};
+
+const Tuning& tuning();
+
+}  // namespace pask

@@ -19,11 +19,21 @@ from . import pask as P
 _ACT = P.ACT
 
 
+class _HostOnly:
+    """Stand-in for a device tensor of a host-only graph: a fake address."""
+
+    def __init__(self, ptr):
+        self._p = ptr
+
+    def data_ptr(self):
+        return self._p
+
+
 class DeviceModel:
     def __init__(self, spec, device="cuda", solutions=None, alloc=True):
         """spec: a workloads.models spec.  solutions: {layer index: kernel id}
         overriding the library's static choice s* for that layer.
-        alloc=False builds the graph with null device pointers (host-only
+        alloc=False builds the graph with placeholder device pointers (host-only
         planning / workspace sizing, no GPU needed)."""
         self.spec = spec
         self.device = device
@@ -36,22 +46,32 @@ class DeviceModel:
         self._tensors = []
         self._nodes = []
         self._keep = []
+        self._blobs = {}      # pointer -> host array of every weight / bias / gamma / beta
+        self._fake_next = self._FAKE
         self._build()
 
     # ------------------------------------------------------------ helpers
     def _dev(self, arr, dtype):
+        host = torch.from_numpy(np.ascontiguousarray(arr)).to(dtype)
         if not self.alloc:
-            self._keep.append(arr)
-            return None
-        t = torch.from_numpy(np.ascontiguousarray(arr)).to(dtype).to(self.device)
+            t = _HostOnly(self._fake(host.numel() * host.element_size()))
+        else:
+            t = host.to(self.device)
+        self._blobs[t.data_ptr()] = host
         self._keep.append(t)
         return t
 
-    _FAKE = 1 << 20   # placeholder address for host-only graphs (never dereferenced)
+    # placeholder addresses for host-only graphs (never dereferenced): distinct,
+    # non-overlapping ranges, so the runtime's aliasing check sees what a real
+    # allocation would give
+    _FAKE = 1 << 40
+
+    def _fake(self, nbytes):
+        p = self._fake_next
+        self._fake_next += (max(nbytes, 1) + 255) // 256 * 256
+        return p
 
     def _ptr(self, t):
-        if not self.alloc:
-            return self._FAKE
         return None if t is None else t.data_ptr()
 
     def _new(self, name, shape, dtype, layout, dims, kind):
@@ -59,7 +79,10 @@ class DeviceModel:
             t = torch.empty(shape, dtype=dtype, device=self.device)
             ptr = t.data_ptr()
         else:
-            t, ptr = None, self._FAKE
+            n = 1
+            for d in (shape if shape is not None else dims):
+                n *= d
+            t, ptr = None, self._fake(n * (4 if dtype == torch.float32 else 2))
         self.t[name] = t
         self.dims[name] = dims
         self.kind[name] = kind

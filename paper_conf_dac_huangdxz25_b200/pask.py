@@ -11,6 +11,9 @@ import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libpask.so")
+# test-only build of the same library plus the fake CUDA driver of
+# include/pask_testing.h (never loaded by the product path)
+TESTING_LIB_PATH = os.path.join(_PKG, "libpask_testing.so")
 
 # ---------------------------------------------------------------- enums (pask.h)
 OK, EINVAL, EUNSUPPORTED, ECUDA, ENOMEM, ESTATE = 0, -1, -2, -3, -4, -5
@@ -57,7 +60,8 @@ class Config(C.Structure):
     _fields_ = [("reuse", C.c_int32), ("search", C.c_int32), ("milestone", C.c_int32),
                 ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
                 ("packaging", C.c_int32), ("interleave", C.c_int32), ("graph", C.c_int32),
-                ("catalog", C.c_int32), ("branches", C.c_int32)]
+                ("catalog", C.c_int32), ("branches", C.c_int32), ("timeline", C.c_int32),
+                ("no_prefault", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -74,7 +78,9 @@ class Stats(C.Structure):
                 ("cold_wall_ns", C.c_uint64), ("infer_count", C.c_uint64), ("launches", C.c_uint64),
                 ("load_done_ns", C.c_uint64), ("infer_entry_ns", C.c_uint64),
                 ("first_launch_ns", C.c_uint64), ("last_launch_ns", C.c_uint64),
-                ("encode_begin_ns", C.c_uint64), ("encode_end_ns", C.c_uint64)]
+                ("encode_begin_ns", C.c_uint64), ("encode_end_ns", C.c_uint64),
+                ("kernel_span_ns", C.c_uint64), ("prefault_ns", C.c_uint64),
+                ("prefault_bytes", C.c_uint64), ("max_cluster", C.c_int32), ("reserved0", C.c_int32)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -84,21 +90,30 @@ EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "
            "pask_infer", "pask_infer_host", "pask_sync", "pask_stats", "pask_kernel_is_loaded",
            "pask_destroy", "pask_last_error", "pask_num_kernels", "pask_kernel_name",
            "pask_kernel_function",
-           "pask_kernel_timeline", "pask_node_times", "pask_promote"]
-TEST_EXPORTS = ["pask_test_fake_driver", "pask_test_fake_log"]   # include/pask_testing.h
+           "pask_kernel_timeline", "pask_node_times", "pask_node_intervals", "pask_promote"]
+TEST_EXPORTS = ["pask_test_fake_driver", "pask_test_fake_log", "pask_test_fake_knob"]   # pask_testing.h
+FAKE_OCCUPANCY, FAKE_CURRENT_DEVICE, FAKE_MAX_CLUSTER_LAUNCHED = 1, 2, 3
 
-_lib = None
+_libs = {}
+_use_testing = False
+
+
+def use_testing_library(enable=True):
+    """Test-only: route lib() (and so every Context created afterwards) to
+    libpask_testing.so, which adds the fake driver hooks of pask_testing.h."""
+    global _use_testing
+    _use_testing = bool(enable)
 
 
 def lib():
     """Load libpask.so (build it first with paper_conf_dac_huangdxz25_b200.build)."""
-    global _lib
-    if _lib is not None:
-        return _lib
-    if not os.path.exists(LIB_PATH):
-        raise RuntimeError(f"{LIB_PATH} is missing: run `python -m paper_conf_dac_huangdxz25_b200."
+    path = TESTING_LIB_PATH if _use_testing else LIB_PATH
+    if path in _libs:
+        return _libs[path]
+    if not os.path.exists(path):
+        raise RuntimeError(f"{path} is missing: run `python -m paper_conf_dac_huangdxz25_b200."
                            "build` (there is no fallback path)")
-    L = C.CDLL(LIB_PATH)
+    L = C.CDLL(path)
     P = C.c_void_p
     sig = {
         "pask_version": (C.c_int, []),
@@ -116,19 +131,22 @@ def lib():
         "pask_kernel_timeline": (C.c_int, [P, C.c_int32, C.POINTER(C.c_uint64),
                                            C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
         "pask_node_times": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int32]),
+        "pask_node_intervals": (C.c_int, [P, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64), C.c_int32]),
         "pask_promote": (C.c_int, [P, C.c_int32, C.POINTER(C.c_int32)]),
         "pask_last_error": (C.c_char_p, []),
-        "pask_test_fake_driver": (C.c_int, [C.c_int32, C.c_int32, C.c_int32]),
-        "pask_test_fake_log": (C.c_int32, [C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.c_int32]),
         "pask_num_kernels": (C.c_int32, []),
         "pask_kernel_name": (C.c_char_p, [C.c_int32]),
         "pask_kernel_function": (C.c_char_p, [C.c_int32, C.c_int32]),
     }
+    if path == TESTING_LIB_PATH:
+        sig["pask_test_fake_driver"] = (C.c_int, [C.c_int32, C.c_int32, C.c_int32])
+        sig["pask_test_fake_log"] = (C.c_int32, [C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.c_int32])
+        sig["pask_test_fake_knob"] = (C.c_int32, [C.c_int32, C.c_int32])
     for name, (res, args) in sig.items():
         f = getattr(L, name)
         f.restype = res
         f.argtypes = args
-    _lib = L
+    _libs[path] = L
     return L
 
 
@@ -138,9 +156,9 @@ class PaskError(RuntimeError):
         self.code = code
 
 
-def _check(rc):
+def _check(rc, L=None):
     if rc != OK:
-        raise PaskError(rc, lib().pask_last_error().decode())
+        raise PaskError(rc, (L or lib()).pask_last_error().decode())
     return rc
 
 
@@ -154,14 +172,20 @@ def function_name(k, packaging):
 
 
 def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,
-           interleave=0, graph=0, catalog=0, branches=0):
+           interleave=0, graph=0, catalog=0, branches=0, timeline=0, no_prefault=0):
     return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph,
-                  catalog, branches)
+                  catalog, branches, timeline, no_prefault)
 
 
 def test_fake_driver(enable=True, load_us=0, fail_kernel=-1):
-    """Test-only (include/pask_testing.h): route new contexts to the fake driver."""
+    """Test-only (include/pask_testing.h, libpask_testing.so): route new contexts
+    to the fake driver.  Call use_testing_library() first."""
     _check(lib().pask_test_fake_driver(1 if enable else 0, load_us, fail_kernel))
+
+
+def test_fake_knob(knob, value=0):
+    """Test-only: set / read a fake-driver knob (pask_test_fake_knob)."""
+    return lib().pask_test_fake_knob(knob, value)
 
 
 def test_fake_log(cap=4096):
@@ -198,7 +222,8 @@ class Context:
 
     def __init__(self, device=0, cfg: Config | None = None):
         self.h = C.c_void_p()
-        _check(lib().pask_create(C.byref(self.h), device, C.byref(cfg) if cfg else None))
+        self.L = lib()   # the library this ctx lives in (product, or the testing build)
+        self._ck(self.L.pask_create(C.byref(self.h), device, C.byref(cfg) if cfg else None))
         self.n_nodes = 0
 
     def load_model(self, graph: Graph, plan=True):
@@ -207,7 +232,7 @@ class Context:
         ``bindings()`` afterwards."""
         self.n_nodes = graph.n_nodes
         self._plan_arr = (Binding * max(graph.n_nodes, 1))()
-        _check(lib().pask_load_model(self.h, C.byref(graph), self._plan_arr))
+        self._ck(self.L.pask_load_model(self.h, C.byref(graph), self._plan_arr))
         return self.bindings() if plan else None
 
     def bindings(self):
@@ -217,47 +242,59 @@ class Context:
     def infer(self, stream=0, inputs=None, outputs=None):
         ip = (C.c_void_p * len(inputs))(*inputs) if inputs else None
         op = (C.c_void_p * len(outputs))(*outputs) if outputs else None
-        _check(lib().pask_infer(self.h, ip, op, C.c_void_p(stream)))
+        self._ck(self.L.pask_infer(self.h, ip, op, C.c_void_p(stream)))
 
     def infer_host(self, host_inputs, host_outputs, stream=0):
         ip = (C.c_void_p * len(host_inputs))(*host_inputs)
         op = (C.c_void_p * len(host_outputs))(*host_outputs)
-        _check(lib().pask_infer_host(self.h, ip, op, C.c_void_p(stream)))
+        self._ck(self.L.pask_infer_host(self.h, ip, op, C.c_void_p(stream)))
 
     def sync(self):
-        _check(lib().pask_sync(self.h))
+        self._ck(self.L.pask_sync(self.h))
 
     def stats(self):
         st = Stats()
-        _check(lib().pask_stats(self.h, C.byref(st)))
+        self._ck(self.L.pask_stats(self.h, C.byref(st)))
         return st.as_dict()
 
     def kernel_is_loaded(self, k):
         v = C.c_int32()
-        _check(lib().pask_kernel_is_loaded(self.h, k, C.byref(v)))
+        self._ck(self.L.pask_kernel_is_loaded(self.h, k, C.byref(v)))
         return bool(v.value)
 
     def kernel_timeline(self, k):
         """(load_ns, ready_ns since load_model entry, lib_ns) of catalog kernel k."""
         a, b, c = C.c_uint64(), C.c_uint64(), C.c_uint64()
-        _check(lib().pask_kernel_timeline(self.h, k, C.byref(a), C.byref(b), C.byref(c)))
+        self._ck(self.L.pask_kernel_timeline(self.h, k, C.byref(a), C.byref(b), C.byref(c)))
         return a.value, b.value, c.value
 
     def promote(self, target_catalog=-1):
         """Idle-interval loading of skipped / specialised solutions."""
         n = C.c_int32()
-        _check(lib().pask_promote(self.h, target_catalog, C.byref(n)))
+        self._ck(self.L.pask_promote(self.h, target_catalog, C.byref(n)))
         return n.value
 
     def node_times(self):
         """Per-node GPU ns of the last instrumented inference (cfg.instrument = 1)."""
         arr = (C.c_uint64 * max(self.n_nodes, 1))()
-        _check(lib().pask_node_times(self.h, arr, self.n_nodes))
+        self._ck(self.L.pask_node_times(self.h, arr, self.n_nodes))
         return list(arr[:self.n_nodes])
+
+    def node_intervals(self):
+        """[(start_ns, end_ns)] per node of the last synced inference of a
+        timeline = 1 context (first CTA start / last CTA end, ns after the
+        inference's first kernel start)."""
+        a = (C.c_uint64 * max(self.n_nodes, 1))()
+        b = (C.c_uint64 * max(self.n_nodes, 1))()
+        self._ck(self.L.pask_node_intervals(self.h, a, b, self.n_nodes))
+        return list(zip(a[:self.n_nodes], b[:self.n_nodes]))
+
+    def _ck(self, rc):
+        return _check(rc, self.L)
 
     def close(self):
         if self.h:
-            _check(lib().pask_destroy(self.h))
+            self._ck(self.L.pask_destroy(self.h))
             self.h = C.c_void_p()
 
     def __del__(self):

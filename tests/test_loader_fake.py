@@ -24,8 +24,10 @@ pytestmark = pytest.mark.timeout(120)
 @pytest.fixture(scope="module", autouse=True)
 def built():
     pbuild.build()
+    P.use_testing_library(True)     # libpask_testing.so: the product library has no fake driver
     yield
     P.test_fake_driver(False)
+    P.use_testing_library(False)
 
 
 MODES = [
@@ -268,3 +270,95 @@ def test_family_variant_covers_the_plan(name, variant):
     expect = os.path.getsize(os.path.join(B.BUILD, f"pask_families_{variant}.fatbin"))
     expect += sum(os.path.getsize(os.path.join(B.BUILD, P.kernel_name(k) + ".fatbin")) for k in own)
     assert st["code_bytes_loaded"] == expect
+
+
+def test_create_refuses_a_context_of_another_device():
+    """pask_create binds `device`'s primary context; a calling thread
+    whose current context belongs to another device is refused (the ctx could not
+    use the caller's device pointers) instead of silently issuing there."""
+    P.test_fake_driver(True)
+    P.test_fake_knob(P.FAKE_CURRENT_DEVICE, 0)
+    with pytest.raises(P.PaskError) as ei:
+        P.Context(1, P.config())
+    assert ei.value.code == P.EINVAL and "device 0" in str(ei.value)
+    ctx = P.Context(0, P.config())            # the current device's ctx is fine
+    ctx.close()
+    P.test_fake_knob(P.FAKE_CURRENT_DEVICE, 1)
+    ctx = P.Context(1, P.config())            # ... and so is device 1 once it is current
+    ctx.close()
+
+
+def test_overlapping_tensors_run_on_one_stream():
+    """branch dependencies are tracked by tensor index, so a graph whose
+    tensors overlap in memory (or that is rebound onto an overlapping buffer)
+    issues everything on one stream."""
+    spec, _ = build_model("resnet50")
+    dm = DeviceModel(spec, alloc=False)
+    P.test_fake_driver(True)
+    ctx = P.Context(0, P.config(branches=1))
+    ctx.load_model(dm.graph)
+    ctx.infer(0)
+    ctx.sync()
+    assert sum(1 for _, kind in P.test_fake_log() if kind == 3) == 4       # ResNet-50 downsample convs
+    # rebind the output (softmax) onto the first activation: the tensors now overlap
+    first_act = dm._tensors[dm.index[spec["layers"][0]["out"]]].dptr
+    P.test_fake_driver(True)
+    ctx.infer(0, outputs=[first_act])
+    ctx.sync()
+    ctx.close()
+    assert sum(1 for _, kind in P.test_fake_log() if kind == 3) == 0
+    # a graph that aliases from the start
+    dm2 = DeviceModel(spec, alloc=False)
+    dm2._tensors[dm2.index[spec["layers"][5]["out"]]].dptr = dm2._tensors[dm2.index[spec["layers"][1]["out"]]].dptr
+    dm2._make_graph(None, 0)
+    P.test_fake_driver(True)
+    ctx = P.Context(0, P.config(branches=1))
+    ctx.load_model(dm2.graph)
+    ctx.infer(0)
+    ctx.sync()
+    ctx.close()
+    assert sum(1 for _, kind in P.test_fake_log() if kind == 3) == 0
+
+
+def test_cluster_size_capped_by_device_occupancy():
+    """the tiny CNN's FC (M = 1, K = 16384) plans a 16-CTA split-K
+    cluster; where the device cannot co-schedule one the node is lowered again
+    with at most 8, before it is launched."""
+    spec, _ = build_model("tiny_cnn")
+    for occ, want in ((1, 16), (0, 8)):
+        P.test_fake_driver(True)
+        P.test_fake_knob(P.FAKE_OCCUPANCY, occ)
+        for mode in (dict(), dict(proactive=1), dict(proactive=0)):
+            P.test_fake_driver(True)
+            P.test_fake_knob(P.FAKE_OCCUPANCY, occ)
+            ctx = P.Context(0, P.config(**mode))
+            ctx.load_model(DeviceModel(spec, alloc=False).graph)
+            ctx.infer(0)
+            ctx.sync()
+            st = ctx.stats()
+            ctx.close()
+            assert st["max_cluster"] == want, mode
+            assert P.test_fake_knob(P.FAKE_MAX_CLUSTER_LAUNCHED) == want, mode
+
+
+def test_timeline_api_states():
+    """cfg.timeline: pask_node_intervals returns one (start, end) per node after a
+    sync (the fake runs no kernel: all zero, busy 0); without timeline it is
+    PASK_ESTATE."""
+    spec, _ = build_model("tiny_cnn")
+    P.test_fake_driver(True)
+    ctx = P.Context(0, P.config(timeline=1))
+    ctx.load_model(DeviceModel(spec, alloc=False).graph)
+    ctx.infer(0)
+    ctx.sync()
+    assert ctx.node_intervals() == [(0, 0)] * len(spec["layers"])
+    assert ctx.stats()["gpu_busy_ns"] == 0
+    ctx.close()
+    ctx = P.Context(0, P.config())
+    ctx.load_model(DeviceModel(spec, alloc=False).graph)
+    ctx.infer(0)
+    ctx.sync()
+    with pytest.raises(P.PaskError) as ei:
+        ctx.node_intervals()
+    assert ei.value.code == P.ESTATE
+    ctx.close()
