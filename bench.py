@@ -3,19 +3,29 @@
 
 Workload (BASELINE.json configs[1]): ResNet-50, batch 1, 224x224, bf16, random
 weights, synthetic N(0,1) input.  A "step" is one inference through the C ABI
-(pask_infer: all 58 layers).  Per process:
+(pask_infer: all 58 layers).  Metric (BASELINE.json): cold first-inference
+latency vs hot; imgs/s per B200; kernels loaded per model.
 
-  cold   pask_load_model entry -> first inference complete (host clock; the
-         paper's cold start: planning + proactive code loading + issue + GPU)
-  hot    K timed inferences, L2 flushed before each (a 256 MiB memset outside
-         the CUDA-event window), mean device time per inference
-  value  imgs/s over all ranks = N * 1000 / max-over-ranks(hot ms)
-  e2e    the same through pask_infer_host: pinned host input -> H2D -> 58
-         kernels -> D2H of the softmax output -> sync, host clock per step
+  value  imgs/s over all ranks = N * batch * 1000 / max-over-ranks(hot ms), hot =
+         K timed inferences replaying the captured CUDA graph, L2 flushed before
+         each (a 256 MiB memset outside the CUDA-event window)
+  cold   SURVEY.md §8(d): >= 20 fresh native processes (pask_cold), each
+         t0 = pask_load_model entry -> t1 = first inference done; median / p90,
+         with and without the host prefault of the code images, and a timeline
+         set (cfg.timeline: per-kernel %globaltimer stamps) for the partitioned
+         breakdown (Fig. 1(b) / Fig. 7) and the cold GPU utilisation (Fig. 6(b))
+  hot    graph replay (value) and direct issue (the cold start's own issue
+         path without loading: the paper's Ideal)
+  e2e    pask_infer_host: pinned host input -> H2D -> the model -> D2H of the
+         outputs -> sync, host clock per step
+  headline  the LAST key of the line: the compact cold / hot / ratio / util /
+         breakdown / kernels block of every config (C1-C4) from this run
 
-N > 1 (torchrun): independent replicas, one process per GPU, cold-starting
-concurrently after a barrier (the path does not shard; no
-data-path collective -- gloo is used only for the barrier and the max).
+N > 1 (torchrun): independent replicas, one process per GPU (SURVEY.md §8(e):
+the path does not shard; no data-path collective -- gloo carries the barrier,
+the max and the gather of the replica statistics).  Every rank cold-starts
+native pask_cold children released together after a barrier (>= 10 trials),
+then rank 0 alone for the same-run cold(1) -> loader contention cold(N)/cold(1).
 
 `--impl reference` times the fp64 numpy oracle (the reference arm of this
 tier) on the host cores, rank 0 only.
@@ -35,6 +45,8 @@ sys.path.insert(0, ROOT)
 
 METRIC = "cold first-inference latency ms vs hot; imgs/s per B200; kernels loaded/model"
 PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+CONFIG_MODELS = ["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base"]   # BASELINE.json configs[0..3]
+BREAKDOWN_KEYS = ["plan", "load", "issue", "gpu_busy", "gpu_idle", "other"]
 
 
 def load_peaks():
@@ -48,8 +60,11 @@ def load_peaks():
 
 # ---------------------------------------------------------------- algorithmic work
 def node_work(spec, li):
-    """(bytes, flops) of layer li: inputs + weights + outputs (+ residual, bias)
-    at their device precision (bf16 tensors, fp32 bias), SURVEY.md §8(d)."""
+    """(bytes, flops) of layer li: bytes = inputs + weights +
+    outputs (+ residual, bias, gamma / beta) at their device precision (bf16
+    tensors, fp32 vectors; the stem reads its input padded to 8 channels, which
+    the kernel really moves); flops = 2 x the multiply-adds of the logical
+    operator (unpadded channels)."""
     L = spec["layers"][li]
     sh = spec["tensors"]
     op = L["op"]
@@ -65,14 +80,14 @@ def node_work(spec, li):
     if op == "conv":
         k, cg, r, s = L["w"].shape
         n, c, h, w = sh[L["inputs"][0]]
-        c_dev = max(8, (c + 7) // 8 * 8) if L["groups"] == 1 else c
+        dense = L["groups"] == 1
+        c_dev = max(8, (c + 7) // 8 * 8) if dense else c
         _, _, p, q = sh[L["out"]]
-        byt = n * h * w * c_dev * 2 + k * r * s * (c_dev if L["groups"] == 1 else 1) * 2 + \
+        byt = n * h * w * c_dev * 2 + k * r * s * (c_dev if dense else 1) * 2 + \
             n * p * q * k * 2 + (k * 4 if L["b"] is not None else 0)
         if L["res"]:
             byt += n * p * q * k * 2
-        flops = 2 * n * p * q * k * (c_dev if L["groups"] == 1 else 1) * r * s
-        return byt, flops
+        return byt, 2 * n * p * q * k * cg * r * s
     if op == "linear":
         m, nout = sh[L["out"]]
         kin = L["w"].shape[1]
@@ -80,9 +95,42 @@ def node_work(spec, li):
         if L["res"]:
             byt += m * nout * 2
         return byt, 2 * m * nout * kin
-    if op == "pool":
-        return numel(L["inputs"][0]) * 2 + numel(L["out"]) * 2, 0
-    return numel(L["inputs"][0]) * 2 + numel(L["out"]) * 2, 0
+    if op == "qk":     # scores[h] = Q_h K_h^T: read Q and K, write the scores
+        heads, dh = L["heads"], L["head_dim"]
+        s_ = sh[L["inputs"][0]][0]
+        return 2 * s_ * heads * dh * 2 + heads * s_ * s_ * 2, 2 * heads * s_ * s_ * dh
+    if op == "pv":     # ctx[:, h] = P_h V_h: read P and V, write the context
+        heads, dh = L["heads"], L["head_dim"]
+        s_ = sh[L["inputs"][1]][0]
+        return heads * s_ * s_ * 2 + s_ * heads * dh * 2 + s_ * heads * dh * 2, 2 * heads * s_ * dh * s_
+    if op == "attention":   # fused: read Q, K, V, write the context
+        heads, dh = L["heads"], L["head_dim"]
+        s_ = sh[L["inputs"][0]][0]
+        return 3 * s_ * heads * dh * 2 + s_ * heads * dh * 2, 4 * heads * s_ * s_ * dh
+    if op == "layernorm":
+        cols = sh[L["inputs"][0]][-1]
+        return numel(L["inputs"][0]) * 2 + numel(L["out"]) * 2 + 2 * cols * 4, 0
+    return numel(L["inputs"][0]) * 2 + numel(L["out"]) * 2, 0   # pool, softmax
+
+
+def step_shares(intervals, kernels):
+    """Partition of one inference's GPU busy time among the catalog solutions,
+    from the timeline stamps of a PDL-chained (graph-replayed) step: in end-time
+    order, node i is charged end_i - max(start_i, latest end before it), the
+    time during which it was the last node to finish.  Charges sum to the busy
+    union.  Returns {kernel: (charged_ns, launches)}."""
+    order = sorted(range(len(intervals)), key=lambda i: intervals[i][1])
+    out, latest = {}, None
+    for i in order:
+        s, e = intervals[i]
+        if e == 0 and s == 0:
+            continue
+        lo = s if latest is None else max(s, latest)
+        ch = max(0, e - lo)
+        latest = e if latest is None else max(latest, e)
+        c, n = out.get(kernels[i], (0, 0))
+        out[kernels[i]] = (c + ch, n + 1)
+    return out
 
 
 # ---------------------------------------------------------------- replicas
@@ -94,6 +142,52 @@ def reduce_max(values, dist=None):
     if dist is not None:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return [float(v) for v in t]
+
+
+def replica_cold_trials(run_waiting_child, dist, rank, trials):
+    """`trials` concurrent cold starts -- every rank starts its
+    child (set up, waiting), a barrier, then each releases its child into the
+    cold window -- and `trials` solo cold starts of rank 0 (the others wait at
+    the barrier) for the same-run cold(1).  run_waiting_child() returns
+    (release, collect): release() lets the child start its cold window,
+    collect() returns its JSON result.  Returns (concurrent, solo) lists of
+    result dicts (solo empty on ranks != 0)."""
+    conc, solo = [], []
+    for _ in range(trials):
+        release, collect = run_waiting_child()
+        dist.barrier()
+        release()
+        conc.append(collect())
+        dist.barrier()
+    for _ in range(trials):
+        if rank == 0:
+            release, collect = run_waiting_child()
+            release()
+            solo.append(collect())
+        dist.barrier()
+    return conc, solo
+
+
+def replica_summary(per_rank_conc, solo, per_rank_hot_ms, batch):
+    """Rank 0's replica block: per-replica cold median / max over the trials,
+    the contention ratio cold(N) / cold(1) (medians, same run), per-replica
+    kernels loaded, and aggregate / per-GPU hot imgs/s."""
+    n = len(per_rank_conc)
+    per = []
+    for r, trials in enumerate(per_rank_conc):
+        c = [t["cold_us"] / 1e3 for t in trials]
+        per.append({"rank": r, "cold_med_ms": round(statistics.median(c), 3), "cold_max_ms": round(max(c), 3),
+                    "trials": len(c), "kernels_loaded": sorted({int(t["kernels_loaded"]) for t in trials})})
+    all_conc = [t["cold_us"] / 1e3 for trials in per_rank_conc for t in trials]
+    solo_ms = [t["cold_us"] / 1e3 for t in solo]
+    cn = statistics.median(all_conc)
+    c1 = statistics.median(solo_ms) if solo_ms else None
+    agg = sum(batch * 1000.0 / h for h in per_rank_hot_ms)
+    return {"n_replicas": n, "cold_N_med_ms": round(cn, 3), "cold_N_max_ms": round(max(all_conc), 3),
+            "cold_1_med_ms": round(c1, 3) if c1 else None,
+            "contention": round(cn / c1, 3) if c1 else None,
+            "per_replica": per, "hot_imgs_s_aggregate": round(agg, 1),
+            "hot_imgs_s_per_gpu": round(agg / n, 1)}
 
 
 # ---------------------------------------------------------------- clocks
@@ -178,7 +272,7 @@ def run_reference(args, spec, x, rank):
         "impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "imgs/s",
         "n_gpus": args.gpus, "steps": len(ts), "warmup": len(w), "ms_per_step": round(1e3 * mean_s, 2),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": {"workload": args.workload_name, "global_batch": 1,
+        "data": "synthetic", "config": {"workload": args.workload_name, "global_batch": args.batch,
                                         "model": args.model},
         "cpu_baseline": {"value": round(val, 4), "unit": "imgs/s", "cores": cores_used(),
                          "kind": "oracle", "cpu": cpu_model(),
@@ -187,6 +281,40 @@ def run_reference(args, spec, x, rank):
                 "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- cold samples (native children)
+def bench_cfg(args, **extra):
+    return {"packaging": args.packaging, "branches": args.branches, "graph": args.graph, **extra}
+
+
+def cold_block(cs, image, cfg, n, n_tl, hot_children):
+    """Fresh-process cold samples of one config: n cold starts, n_tl timeline
+    cold starts (breakdown + utilisation), and optionally hot children (graph
+    replay and direct issue, L2 flushed, 200 inferences each)."""
+    samples = cs.sample(image, cfg, n)
+    tl = cs.sample(image, {**cfg, "timeline": 1}, n_tl) if n_tl else []
+    out = {"cold": cs.summarize(samples), "breakdown": cs.breakdown(tl) if tl else None,
+           "plan": [samples[0]["queries"], samples[0]["hits"], samples[0]["lookups"]],
+           "launches": samples[0]["launches"], "load_timeline_us": samples[0]["timeline"]}
+    if tl:
+        out["cold_timeline_med_us"] = statistics.median(s["cold_us"] for s in tl)
+    if hot_children:
+        out["hot_graph_us"] = cs.run_child(image, {**cfg, "graph": 1}, hot=200)["hot_median_us"]
+        out["hot_direct_us"] = cs.run_child(image, {**cfg, "graph": 0}, hot=200)["hot_median_us"]
+    return out
+
+
+def headline_entry(cold_ms, p90_ms, n, hot_graph_ms, hot_direct_ms, bd, kernels, launches, extra=None):
+    e = {"cold_ms": [round(cold_ms, 3), round(p90_ms, 3), n],
+         "hot_ms": [round(hot_graph_ms, 4), round(hot_direct_ms, 4)],
+         "cold/hot": [round(cold_ms / hot_graph_ms, 2), round(cold_ms / hot_direct_ms, 2)],
+         "util": bd["util"] if bd else None,
+         "bd_us": [round(bd[k]) for k in BREAKDOWN_KEYS] if bd else None,
+         "kernels": int(kernels), "launches": int(launches)}
+    if extra:
+        e.update(extra)
+    return e
 
 
 # ---------------------------------------------------------------- main
@@ -200,11 +328,16 @@ def main():
                     choices=["tiny_cnn", "resnet50", "mobilenet_v2", "bert_base", "bert_base_fa"])
     ap.add_argument("--batch", type=int, default=1, help="images per inference (Table II sweep)")
     ap.add_argument("--branches", type=int, default=1, choices=[0, 1],
-                    help="1 (default): independent nodes (ResNet downsample convs) on a second stream in "
-                         "the hot graph (DESIGN.md D9)")
+                    help="1 (default): independent nodes (ResNet downsample convs) on a second stream "
+                         "(DESIGN.md D9)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cold-samples", type=int, default=4,
-                    help="extra fresh-process cold starts (N = 1); cold_over_hot uses the median")
+    ap.add_argument("--cold-samples", type=int, default=20,
+                    help="fresh-process cold starts per config (native pask_cold children)")
+    ap.add_argument("--timeline-samples", type=int, default=10,
+                    help="fresh-process cold starts with cfg.timeline (breakdown, GPU utilisation)")
+    ap.add_argument("--no-configs", action="store_true",
+                    help="skip the other configs' compact block (C1-C4 headline)")
+    ap.add_argument("--replica-trials", type=int, default=10, help="N > 1: concurrent cold-start trials")
     ap.add_argument("--no-flush", action="store_true", help="L2-warm hot loop (reported as such)")
     ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
                     help="1: hot inferences replay a CUDA graph captured on the 2nd call")
@@ -221,6 +354,8 @@ def main():
         "bert_base_fa": "BERT-base seq 128 batch 1 cold start, attention fused (QK^T -> softmax -> PV "
                         "in one kernel; SURVEY.md 8(f) NEXT #4)",
     }[args.model]
+    if args.batch != 1:
+        args.workload_name += f" (Table II sweep: batch {args.batch})"
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -245,6 +380,7 @@ def main():
     from paper_conf_dac_huangdxz25_b200 import build as pbuild
     from paper_conf_dac_huangdxz25_b200 import pask as P
     from paper_conf_dac_huangdxz25_b200.model import DeviceModel
+    from scripts import cold_samples as cs
 
     pbuild.build()
     torch.cuda.set_device(local_rank)
@@ -267,24 +403,15 @@ def main():
         if dist:
             dist.barrier()
 
-    # ---------------- cold: pask_load_model entry -> first inference done
+    # ---------------- in-process cold: pask_load_model entry -> first inference done
     barrier()
     torch.cuda.synchronize()
-    t0 = time.perf_counter_ns()
     ctx.load_model(dm.graph, plan=False)
     ctx.infer(sp)
     ctx.sync()
-    t1 = time.perf_counter_ns()
     plan = ctx.bindings()
     cold_stats = ctx.stats()
-    cold_ms = cold_stats["cold_wall_ns"] / 1e6      # library clock: load_model entry -> sync return
-    cold_py_ms = (t1 - t0) / 1e6                    # the same window seen from Python
-    timeline = {}
-    for k in range(P.num_kernels()):
-        ld, rd, lb = ctx.kernel_timeline(k)
-        if ld:
-            timeline[P.kernel_name(k)] = {"load_us": round(ld / 1e3, 1), "ready_at_us": round(rd / 1e3, 1),
-                                          "lib_us": round(lb / 1e3, 1)}
+    cold_inproc_ms = cold_stats["cold_wall_ns"] / 1e6
     solutions = sorted(P.kernel_name(k) for k in {b[2] for b in plan})  # Algorithm 1's bound set
     loaded = sorted({P.function_name(k, args.packaging) for k in range(P.num_kernels())
                      if ctx.kernel_is_loaded(k)})                       # CUfunctions resident
@@ -315,6 +442,7 @@ def main():
     clocks = sampler.stop()
     step_ms = [a.elapsed_time(b) for a, b in ev]
     hot_ms = statistics.mean(step_ms)
+    hot_med_ms = statistics.median(step_ms)
 
     # ---------------- L2-warm back-to-back (context: serving the same model repeatedly)
     torch.cuda.synchronize()
@@ -345,9 +473,9 @@ def main():
             e2e_s.append(b - a)
     e2e_ms = 1e3 * statistics.mean(e2e_s)
 
-    # ---------------- hot through the direct-issue path (SURVEY.md §8(d) protocol:
-    # the paper's "Ideal", PAPER.md:178 -- the cold start's own issue path without
-    # any loading), L2 flushed like the timed loop; a separate context, graph off
+    # ---------------- hot through the direct-issue path (the paper's
+    # "Ideal", PAPER.md:178 -- the cold start's own issue path without any loading),
+    # L2 flushed like the timed loop; a separate context, graph off
     if args.graph:
         dctx = P.Context(local_rank, P.config(packaging=args.packaging, graph=0, branches=args.branches))
         dctx.load_model(dm.graph, plan=False)
@@ -365,14 +493,33 @@ def main():
             b_.record(stream)
             dev_.append((a_, b_))
         torch.cuda.synchronize()
-        hot_direct_ms = statistics.mean(a_.elapsed_time(b_) for a_, b_ in dev_)
+        d_ms = [a_.elapsed_time(b_) for a_, b_ in dev_]
+        hot_direct_ms = statistics.mean(d_ms)
+        hot_direct_med_ms = statistics.median(d_ms)
         dctx.close()
     else:
-        hot_direct_ms = hot_ms
+        hot_direct_ms, hot_direct_med_ms = hot_ms, hot_med_ms
 
-    # ---------------- per-kernel roofline: instrumented pass (separate context)
+    # ---------------- per-kernel roofline: each solution's share of the step from
+    # the timeline stamps of graph-replayed, PDL-chained steps (a separate context,
+    # cfg.timeline), times the event-timed hot step
+    tctx = P.Context(local_rank, P.config(packaging=args.packaging, graph=args.graph, branches=args.branches,
+                                          timeline=1))
+    tctx.load_model(dm.graph, plan=False)
+    kern_of = [b[2] for b in plan]
+    charged = {}
+    for r in range(12):
+        flush()
+        tctx.infer(sp)
+        tctx.sync()
+        if r >= 2:
+            for k, (c, nl) in step_shares(tctx.node_intervals(), kern_of).items():
+                cc, nn = charged.get(k, (0, 0))
+                charged[k] = (cc + c, nn + nl)
+    tctx.close()
+    # ... and the isolated per-launch figure (events around each node, no PDL overlap)
     ictx = P.Context(local_rank, P.config(instrument=1))
-    iplan = ictx.load_model(dm.graph)
+    ictx.load_model(dm.graph)
     reps = 10
     acc = [0] * n_nodes
     for r in range(reps + 2):
@@ -381,86 +528,126 @@ def main():
         ictx.sync()
         if r >= 2:
             acc = [a + b for a, b in zip(acc, ictx.node_times())]
-    node_ms = [a / reps / 1e6 for a in acc]
+    iso_ms = [a / reps / 1e6 for a in acc]
     ictx.close()
     per_kernel = {}
-    for (i, want, bound, how, lk), t in zip(plan, node_ms):
+    for (i, want, bound, how, lk), t in zip(plan, iso_ms):
         byt, fl = node_work(spec, i)
-        d = per_kernel.setdefault(P.kernel_name(bound), {"launches": 0, "ms": 0.0, "bytes": 0, "flops": 0})
+        d = per_kernel.setdefault(bound, {"launches": 0, "iso_ms": 0.0, "bytes": 0, "flops": 0})
         d["launches"] += 1
-        d["ms"] += t
+        d["iso_ms"] += t
         d["bytes"] += byt
         d["flops"] += fl
-    dom = max(per_kernel, key=lambda k: per_kernel[k]["ms"])
+    tot_charged = sum(c for c, _ in charged.values()) or 1
+    for k, d in per_kernel.items():
+        d["share"] = charged.get(k, (0, 0))[0] / tot_charged
+        d["step_ms"] = d["share"] * hot_ms
+    dom = max(per_kernel, key=lambda k: per_kernel[k]["step_ms"])
     peaks, peak_src = load_peaks()
     dk = per_kernel[dom]
-    # the kernel's time inside the timed step: its share of the instrumented
-    # per-node times (the ncu launch list gives the same share) x the timed
-    # region's event-measured step time; the isolated per-launch time (events
-    # around each node, no PDL overlap) is reported beside it
-    share = dk["ms"] / sum(v["ms"] for v in per_kernel.values())
-    in_step_ms = share * hot_ms
-    gbs = dk["bytes"] / (in_step_ms * 1e-3) / 1e9
-    tfl = dk["flops"] / (in_step_ms * 1e-3) / 1e12
-    gbs_iso = dk["bytes"] / (dk["ms"] * 1e-3) / 1e9
-    # every solution's bandwidth inside the step (same share method): the
-    # memory-bound ones against HBM, the contractions with their tensor rate too
-    tot_ms = sum(v["ms"] for v in per_kernel.values())
+    gbs = dk["bytes"] / (dk["step_ms"] * 1e-3) / 1e9
+    tfl = dk["flops"] / (dk["step_ms"] * 1e-3) / 1e12
+    gbs_iso = dk["bytes"] / (dk["iso_ms"] * 1e-3) / 1e9
     per_kernel_roofline = {}
     for k, v in per_kernel.items():
-        st_ms = v["ms"] / tot_ms * hot_ms
-        per_kernel_roofline[k] = {
+        st_ms = max(v["step_ms"], 1e-9)
+        per_kernel_roofline[P.kernel_name(k)] = {
             "launches": v["launches"], "bytes_per_launch": int(v["bytes"] / v["launches"]),
             "in_step_us_per_launch": round(1e3 * st_ms / v["launches"], 2),
+            "share": round(v["share"], 4),
             "achieved_gbs": round(v["bytes"] / (st_ms * 1e-3) / 1e9, 1),
             "frac_hbm": round(v["bytes"] / (st_ms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4),
-            "tflops": round(v["flops"] / (st_ms * 1e-3) / 1e12, 2)}
+            "tflops": round(v["flops"] / (st_ms * 1e-3) / 1e12, 2),
+            "isolated_us_per_launch": round(1e3 * v["iso_ms"] / v["launches"], 2)}
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "dram_traffic.json")
     if os.path.exists(tpath):
         with open(tpath) as f:
-            traffic = json.load(f).get(args.model, {}).get(dom)
+            traffic = json.load(f).get(args.model, {}).get(P.kernel_name(dom))
     roofline = {"bound": "hbm", "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": traffic,
-                "kernel": dom, "launches_per_step": dk["launches"],
+                "kernel": P.kernel_name(dom), "launches_per_step": dk["launches"],
                 "algorithmic_bytes_per_launch": int(dk["bytes"] / dk["launches"]),
-                "avg_launch_us": round(1e3 * in_step_ms / dk["launches"], 2),
-                "share_of_step": round(share, 4),
-                "method": "achieved = algorithmic bytes / (share of the step x timed hot step time); share "
-                          "from per-node CUDA events of an instrumented pass",
-                "isolated": {"avg_launch_us": round(1e3 * dk["ms"] / dk["launches"], 2),
+                "avg_launch_us": round(1e3 * dk["step_ms"] / dk["launches"], 2),
+                "share_of_step": round(dk["share"], 4),
+                "method": "achieved = algorithmic bytes / (share of the step x event-timed hot step); share = "
+                          "the kernel's charge of the busy time in graph-replayed PDL steps (timeline stamps)",
+                "isolated": {"avg_launch_us": round(1e3 * dk["iso_ms"] / dk["launches"], 2),
                              "achieved": round(gbs_iso, 1), "frac": round(gbs_iso / peaks["hbm_gbs"], 4),
                              "how": "events around each node, no PDL overlap (launch + prologue exposed)"},
                 "tensor_tflops": round(tfl, 2),
                 "tensor_frac_of_bf16_burst": round(tfl / peaks["bf16_tflops"], 4),
                 "peak_source": f"{peak_src} (MEASURED_PEAKS.json hbm_gbs / bf16_tflops)",
                 "l2": "flushed before each inference (weights from HBM)"}
+    ctx.close()
+
+    # ---------------- N > 1: concurrent replica cold starts (native children)
+    replicas = None
+    if world > 1:
+        image = cs.write_image(args.model, batch=args.batch)
+        cfg = bench_cfg(args)
+
+        def waiting_child():
+            p = subprocess.Popen([cs.EXE, image, "--cfg", cs.cfg_arg(cfg), "--device", str(local_rank),
+                                  "--wait"], stdin=subprocess.PIPE, stdout=subprocess.PIPE,
+                                 stderr=subprocess.PIPE, text=True)
+            if p.stdout.readline().strip() != "ready":
+                raise RuntimeError("replica child failed: " + p.stderr.read()[-2000:])
+
+            def release():
+                p.stdin.write("go\n")
+                p.stdin.flush()
+
+            def collect():
+                so, se = p.communicate(timeout=120)
+                return json.loads([l for l in so.splitlines() if l.startswith("{")][-1])
+            return release, collect
+        conc, solo = replica_cold_trials(waiting_child, dist, rank, args.replica_trials)
+        os.unlink(image)
+        gathered = [None] * world
+        dist.all_gather_object(gathered, {"conc": conc, "solo": solo, "hot_ms": hot_ms})
+        if rank == 0:
+            replicas = replica_summary([g["conc"] for g in gathered], gathered[0]["solo"],
+                                       [g["hot_ms"] for g in gathered], args.batch)
 
     # ---------------- max over ranks
-    hot_max, cold_max, e2e_max, warm_max, direct_max = reduce_max(
-        [hot_ms, cold_ms, e2e_ms, hot_warm_ms, hot_direct_ms], dist)
-    ctx.close()
+    hot_max, e2e_max, warm_max, direct_max = reduce_max([hot_ms, e2e_ms, hot_warm_ms, hot_direct_ms], dist)
     if rank != 0:
         if dist:
             dist.destroy_process_group()
         return
 
-    # ---------------- more cold samples, each a fresh process (N = 1 only: with
-    # replicas the ranks' own cold starts are the concurrent measurement)
-    fresh = []
-    if args.cold_samples > 0 and world == 1:
-        scheme = ["pask", "pask_single_image", "pask_families", "pask_single_function"][args.packaging]
-        if args.branches and args.packaging == 2:
-            scheme = "pask_families_branches"  # the same pask_config as this process's context
-        for _ in range(args.cold_samples):
-            r = subprocess.run([sys.executable, os.path.join(ROOT, "scripts", "cold_samples.py"), "--model",
-                                args.model, "--child", scheme, "--batch", str(args.batch)],
-                               capture_output=True, text=True, timeout=300)
-            js = [l for l in r.stdout.splitlines() if l.startswith("{")]
-            if js:
-                fresh.append(json.loads(js[-1])["cold_us"] / 1e3)
-    colds = sorted([cold_max] + fresh)
-    cold_med = statistics.median(colds)
+    # ---------------- cold in fresh native processes (N = 1; with replicas the
+    # concurrent trials above are the measurement)
+    headline, configs_detail, main_cold = {}, {}, None
+    if world == 1 and args.cold_samples > 0:
+        cfg = bench_cfg(args)
+        image = cs.write_image(args.model, batch=args.batch)
+        try:
+            main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
+            nopf = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1}, args.cold_samples))
+            main_cold["cold_no_prefault"] = nopf
+        finally:
+            os.unlink(image)
+        c = main_cold["cold"]
+        headline[args.model] = headline_entry(
+            c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"], hot_max, direct_max, main_cold["breakdown"],
+            c["kernels_loaded"], main_cold["launches"],
+            {"nopf_ms": [round(nopf["median_us"] / 1e3, 3), round(nopf["p90_us"] / 1e3, 3)]})
+        if not args.no_configs and args.batch == 1:
+            for m in CONFIG_MODELS:
+                if m == args.model:
+                    continue
+                image = cs.write_image(m)
+                try:
+                    blk = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, True)
+                finally:
+                    os.unlink(image)
+                configs_detail[m] = blk
+                c = blk["cold"]
+                headline[m] = headline_entry(c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"],
+                                             blk["hot_graph_us"] / 1e3, blk["hot_direct_us"] / 1e3,
+                                             blk["breakdown"], c["kernels_loaded"], blk["launches"])
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
@@ -489,42 +676,13 @@ def main():
                    "packaging": ["one code object per kernel", "single code object",
                                  "operator families (memory-bound + contraction)",
                                  "single function (both families behind one entry)"][args.packaging],
-                   "branches": "independent nodes on a second stream in the hot graph" if args.branches
-                               else "one stream",
+                   "branches": "independent nodes on a second stream" if args.branches else "one stream",
                    "hot_issue": "CUDA graph replay (captured on the 2nd inference)" if args.graph
                                 else "direct cuLaunchKernelEx per layer",
                    "l2": "warm (no flush)" if args.no_flush else
-                         "flushed (256 MiB memset) before every timed inference"},
-        "cold_ms": round(cold_max, 3),
-        "cold_ms_python_clock": round(cold_py_ms, 3),
-        "hot_ms": round(hot_max, 4),
-        "cold_over_hot": round(cold_med / hot_max, 3),
-        "cold_samples_ms": {"median": round(cold_med, 3), "n": len(colds),
-                            "values": [round(c, 3) for c in colds],
-                            "how": "this process's cold start plus fresh-process samples "
-                                   "(scripts/cold_samples.py child, same model / packaging); "
-                                   "cold_over_hot uses the median"},
-        "hot_l2_warm_ms": round(warm_max, 4),
-        "hot_direct_ms": round(direct_max, 4),
-        "cold_over_hot_direct": round(cold_med / direct_max, 3),
-        "hot_direct_how": "direct cuLaunchKernelEx per layer (the cold start's issue path, no loading: the "
-                          "paper's Ideal, SURVEY.md §8(d)), L2 flushed, separate context",
-        "kernels_loaded": st["kernels_loaded"],
-        "kernels_loaded_names": loaded,
-        "solutions_bound": solutions,
-        "code_objects_loaded": st["code_objects_loaded"],
-        "plan": {"queries": st["queries"], "hits": st["hits"], "lookups": st["lookups"],
-                 "reused_nodes": sum(1 for b in plan if b[3] == 1)},
-        "cold_breakdown_us": {"plan": round(st["plan_ns"] / 1e3, 1),
-                              "encode": round(st["encode_ns"] / 1e3, 1),
-                              "load_total": round(st["load_ns"] / 1e3, 1),
-                              "load_exposed": round(st["load_exposed_ns"] / 1e3, 1),
-                              "issue": round(st["issue_ns"] / 1e3, 1),
-                              "gpu_span": round(st["gpu_span_ns"] / 1e3, 1),
-                              "cold_wall": round(st["cold_wall_ns"] / 1e3, 1)},
-        "load_timeline_us": timeline,
-        "per_kernel_ms": {k: round(v["ms"], 4) for k, v in per_kernel.items()},
-        "per_kernel_roofline": per_kernel_roofline,
+                         "flushed (256 MiB memset) before every timed inference",
+                   "cold": f"{args.cold_samples} fresh native processes per config (pask_cold), "
+                           "t0 = pask_load_model entry, t1 = first inference done"},
         "e2e": {"value": round(world * args.batch * 1000.0 / e2e_max, 2), "unit": "imgs/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": round(e2e_max, 4)},
@@ -533,7 +691,29 @@ def main():
         "cpu_baseline": cpu,
         "clocks": clocks,
         "wall_s_timed_region": round(w1 - w0, 4),
+        "hot_ms": round(hot_max, 4),
+        "hot_median_ms": round(hot_med_ms, 4),
+        "hot_l2_warm_ms": round(warm_max, 4),
+        "hot_direct_ms": round(direct_max, 4),
+        "hot_direct_median_ms": round(hot_direct_med_ms, 4),
+        "cold_inprocess_ms": round(cold_inproc_ms, 3),
+        "kernels_loaded_names": loaded,
+        "solutions_bound": solutions,
+        "code_objects_loaded": st["code_objects_loaded"],
+        "plan": {"queries": st["queries"], "hits": st["hits"], "lookups": st["lookups"],
+                 "reused_nodes": sum(1 for b in plan if b[3] == 1)},
+        "per_kernel_roofline": per_kernel_roofline,
+        "cold_detail": main_cold,
+        "configs_detail": configs_detail or None,
     }
+    # the LAST keys of the line (the driver keeps the tail of stdout): the
+    # replica block (N > 1) or the compact per-config cold / hot block (N = 1)
+    if replicas:
+        line["replicas"] = replicas
+    if headline:
+        line["headline"] = {"legend": {"cold_ms": "med,p90,n", "hot_ms": "graph,direct", "cold/hot": "graph,direct",
+                                       "util": "busy/cold", "bd_us": "/".join(BREAKDOWN_KEYS)},
+                            **headline}
     print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

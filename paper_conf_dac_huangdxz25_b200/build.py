@@ -27,6 +27,8 @@ HOST_SRC = [os.path.join(CSRC, "runtime", f) for f in ("pask.cpp", "plan.cpp", "
 # test-only library libpask_testing.so, never into the product libpask.so
 TEST_SRC = [os.path.join(CSRC, "runtime", "fake_driver.cpp")]
 TEST_LIB = os.path.join(PKG, "libpask_testing.so")
+COLD_SRC = os.path.join(CSRC, "tools", "pask_cold.cpp")
+COLD_EXE = os.path.join(PKG, "pask_cold")   # native cold-start sampler (scripts/cold_samples.py)
 HOST_DEPS = HOST_SRC + TEST_SRC + [os.path.join(CSRC, "runtime", f) for f in
                                    ("plan.h", "driver.h", "tuning.h", "exports.map")] + [
     os.path.join(CSRC, "kernels", "pask_params.h"),
@@ -219,6 +221,13 @@ def _build_locked(force: bool, verbose: bool) -> str:
             _run([cxx, "-shared", "-o", tmp, *[objs[x] for x in srcs], fobj, "-ldl", "-lpthread",
                   "-Wl,--no-undefined", "-Wl,--version-script=" + os.path.join(CSRC, "runtime", "exports.map")])
             shutil.move(tmp, lib)
+    if force or _stale(COLD_EXE, [LIB, COLD_SRC, os.path.join(os.path.dirname(PKG), "include", "pask.h")]):
+        # the native fresh-process cold-start sampler (links libpask.so, dlopens libcuda)
+        cxx = os.environ.get("CXX", "g++")
+        tmp = COLD_EXE + ".tmp"
+        _run([cxx, "-O2", "-std=c++17", "-Wall", f"-I{CUDA}/include", COLD_SRC, "-o", tmp, f"-L{PKG}", "-lpask",
+              "-ldl", "-Wl,-rpath,$ORIGIN"])
+        shutil.move(tmp, COLD_EXE)
     return LIB
 
 

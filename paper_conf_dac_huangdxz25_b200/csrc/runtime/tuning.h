@@ -1,13 +1,13 @@
 // Tiling and issue constants of the runtime, and the experiment switches used
 // to measure the alternatives DESIGN.md reports.
 //
-// Release builds use the constants below.  A build with -DPASK_EXPERIMENTS
-// (PASK_NVCC_DEFINES="-DPASK_EXPERIMENTS" python -m paper_conf_dac_huangdxz25_b200.build)
-// also reads the PASK_* environment variables, ONCE (the first call of tuning(),
-// from pask_create / pask_plan on the caller's thread), and clamps every value
-// to the range the kernels support -- e.g. splits <= min(16, num_kb) is kept by
-// gemm_tiling regardless of PASK_SPLIT_MAX, and the device trace pointer is
-// only honoured in experiment builds.
+// The PASK_* environment variables are read ONCE -- the first tuning() call,
+// from pask_create / pask_plan on the caller's thread, never from the helper
+// thread -- and every value is clamped to the range the kernels support (e.g.
+// splits <= min(16, num_kb) holds in gemm_tiling whatever PASK_SPLIT_MAX says).
+// The device phase trace (PASK_TRACE_PTR: a device address the kernels write
+// to) is honoured only in builds with -DPASK_EXPERIMENTS
+// (PASK_NVCC_DEFINES="-DPASK_EXPERIMENTS" python -m paper_conf_dac_huangdxz25_b200.build).
 #pragma once
 #include <stdint.h>
 

@@ -239,6 +239,67 @@ class DeviceModel:
                              len(self.inputs), self._i_arr, len(self.outputs), self._o_arr,
                              ws, ws_bytes)
 
+    # ------------------------------------------------------------ model image
+    def save_image(self, path, x):
+        """Write the lowered model as a model image for the native cold-start
+        sampler (csrc/tools/pask_cold.cpp): header, the pask_tensor and
+        pask_node arrays (device pointers replaced by blob ids, 1-based, 0 =
+        none), the graph inputs / outputs, and the blobs -- every weight, bias,
+        gamma, beta, and the input x in its device dtype.  Works for host-only
+        graphs (alloc=False) too: no GPU is needed to write it."""
+        import struct
+        blobs, ids = [], {}
+
+        def blob(ptr):
+            if not ptr:
+                return 0
+            if ptr not in ids:
+                ids[ptr] = len(blobs)
+                h = self._blobs[ptr].contiguous()
+                blobs.append(h.view(torch.uint8).numpy().tobytes())
+            return ids[ptr] + 1
+
+        nodes = (P.Node * len(self._nodes))()
+        for i, nd in enumerate(self._nodes):
+            C.memmove(C.byref(nodes[i]), C.byref(nd), C.sizeof(P.Node))
+            for f in ("w", "bias", "gamma", "beta"):
+                setattr(nodes[i], f, blob(getattr(nd, f)) or None)
+        tensors = (P.Tensor * len(self._tensors))()
+        for i, t in enumerate(self._tensors):
+            C.memmove(C.byref(tensors[i]), C.byref(t), C.sizeof(P.Tensor))
+            tensors[i].dptr = None
+        (name, _, _), = self.spec["inputs"]
+        dt = torch.float32 if self._tensors[self.index[name]].dtype == P.F32 else torch.bfloat16
+        xin = torch.from_numpy(np.ascontiguousarray(x)).to(dt)
+        input_blobs = [len(blobs)]
+        blobs.append(xin.view(torch.uint8).numpy().tobytes())
+        with open(path, "wb") as f:
+            f.write(b"PASKMDL1")
+            f.write(struct.pack("<6i", 1, len(self._tensors), len(self._nodes), len(self.inputs),
+                                len(self.outputs), len(blobs)))
+            f.write(struct.pack("<3Q", C.sizeof(P.Tensor), C.sizeof(P.Node), self.ws_bytes or 0))
+            f.write(bytes(tensors))
+            f.write(bytes(nodes))
+            f.write(struct.pack(f"<{len(self.inputs)}i", *self.inputs))
+            f.write(struct.pack(f"<{len(self.outputs)}i", *self.outputs))
+            f.write(struct.pack(f"<{len(input_blobs)}i", *input_blobs))
+            f.write(struct.pack(f"<{len(blobs)}Q", *[len(b) for b in blobs]))
+            for b in blobs:
+                f.write(b)
+                f.write(b"\0" * ((-len(b)) % 256))
+        return path
+
+    def tensor_layout(self):
+        """[(name, torch dtype, device shape, bytes)] in tensor order: how the
+        native sampler's --dump file is laid out."""
+        out = []
+        names = sorted(self.index, key=self.index.get)
+        for nm in names:
+            t = self._tensors[self.index[nm]]
+            nbytes = t.n * t.h * t.w * t.c * (4 if t.dtype == P.F32 else 2)
+            out.append((nm, torch.float32 if t.dtype == P.F32 else torch.bfloat16, nbytes))
+        return out
+
     # ------------------------------------------------------------ data movement
     def set_input(self, x):
         (name, _, dtype), = self.spec["inputs"]

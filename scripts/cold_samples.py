@@ -1,100 +1,153 @@
-"""Cold-start samples in fresh processes (SURVEY.md §8(d) protocol).
+"""Cold-start samples in fresh native processes (SURVEY.md §8(d) protocol).
 
-Each sample is a new Python process: import torch, create the context, upload
-weights, synchronise, pask_create (all outside the window), then
-t0 = pask_load_model entry, t1 = first inference complete.  The parent prints
-the median / p90 per scheme and the paper's breakdown (Fig. 1(b) / Fig. 7
-analog: loading exposed / issue / GPU / other).
+Each sample is a new process of the native sampler
+(paper_conf_dac_huangdxz25_b200/pask_cold, csrc/tools/pask_cold.cpp): it
+creates the context, uploads the weights and the input, synchronises and calls
+pask_create, all outside the window; then t0 = pask_load_model entry and t1 =
+the first inference complete (the library's cold_wall_ns).  The parent writes
+the lowered model once as a model image (DeviceModel.save_image) and runs the
+children; no child imports Python or PyTorch, so a sample costs ~0.1-0.5 s.
 
     python scripts/cold_samples.py --model resnet50 --n 20 [--schemes pask,pask_i,...]
+
+Also the replica harness of SURVEY.md §8(e): N children cold-starting
+together (each prints "ready" and waits for a line on stdin; the parent
+releases them at once), on one GPU (--replicas) or one per GPU.
 """
+from __future__ import annotations
+
 import argparse
 import json
 import os
 import statistics
 import subprocess
 import sys
-import time
+import tempfile
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+EXE = os.path.join(ROOT, "paper_conf_dac_huangdxz25_b200", "pask_cold")
 
-# scheme -> pask_config keywords
+# scheme -> pask_config fields
 SCHEMES = {
-    "pask": dict(),                                   # default: caller uploads, helper encodes
-    "pask_thread": dict(proactive=1),                 # async loader thread
+    "pask": dict(),                                      # library default: caller uploads, helper encodes
+    "pask_thread": dict(proactive=1),                    # async loader thread
     "pask_interleave": dict(proactive=1, interleave=1),  # Fig. 5 interleaving
-    "pask_single_image": dict(packaging=1),           # whole catalog as one code object
-    "pask_families": dict(packaging=2),               # operator families (D8)
-    "pask_single_function": dict(packaging=3),        # both families in one CUfunction (D10)
+    "pask_single_image": dict(packaging=1),              # whole catalog as one code object
+    "pask_families": dict(packaging=2),                  # operator families (D8)
+    "pask_single_function": dict(packaging=3),           # both families in one CUfunction (D10)
     "pask_families_branches": dict(packaging=2, branches=1),  # bench default: + side stream (D9)
-    "pask_families_branches_1s": dict(packaging=2, branches=1),  # ... cold issue on one stream
-    "pask_families_branches_noevw": dict(packaging=2, branches=1),  # ... events not warmed at create
-    "pask_i": dict(reuse=0),                          # PaSK-I: proactive, no reuse
-    "pask_r": dict(search=1),                         # PaSK-R: naive (exhaustive-order) search
-    "reactive": dict(proactive=0, reuse=0),           # Baseline analog: lazy load at first launch
-    "reactive_reuse": dict(proactive=0),              # reuse without the proactive loader
+    "pask_i": dict(reuse=0),                             # PaSK-I: proactive, no reuse
+    "pask_r": dict(search=1),                            # PaSK-R: naive (exhaustive-order) search
+    "reactive": dict(proactive=0, reuse=0),              # Baseline analog: lazy load at first launch
+    "reactive_reuse": dict(proactive=0),                 # reuse without the proactive loader
     # tuned library (per-problem specialised conv solutions)
     "baseline_tuned": dict(catalog=1, proactive=0, reuse=0),  # the paper's Baseline
-    "pask_tuned": dict(catalog=1),                    # PASK over the tuned library
-    "pask_encfirst": dict(),                          # experiment: caller encodes, then uploads
+    "pask_tuned": dict(catalog=1),                       # PASK over the tuned library
 }
-SCHEME_ENV = {"pask_encfirst": {"PASK_ENCODE_FIRST": "1"},
-              "pask_families_branches_1s": {"PASK_DIRECT_ONE_STREAM": "1"},
-              "pask_families_branches_noevw": {"PASK_NO_EVENT_WARM": "1"}}
 
 
-def child(model, scheme, batch=1):
-    import torch
+def cfg_arg(cfg: dict) -> str:
+    return ",".join(f"{k}={int(v)}" for k, v in sorted(cfg.items())) or "reuse=1"
 
-    from paper_conf_dac_huangdxz25_b200 import pask as P
+
+def write_image(model: str, path: str | None = None, batch: int = 1) -> str:
+    """The lowered model + weights + seeded input as a model image (host only)."""
     from paper_conf_dac_huangdxz25_b200.model import DeviceModel
     from workloads import build_model
     spec, x = build_model(model, **({"batch": batch} if batch != 1 else {}))
-    dm = DeviceModel(spec)
-    dm.set_input(x)
-    torch.cuda.synchronize()
-    ctx = P.Context(0, P.config(**SCHEMES[scheme]))
-    s = torch.cuda.current_stream().cuda_stream
-    time.sleep(float(os.environ.get("PASK_COLD_SLEEP_MS", "50")) / 1e3)  # idle before the cold window
-    torch.cuda.synchronize()
-    t0 = time.perf_counter_ns()
-    ctx.load_model(dm.graph, plan=False)
-    ctx.infer(s)
-    ctx.sync()
-    t1 = time.perf_counter_ns()
-    st = ctx.stats()
-    tl = {}
-    for k in range(P.num_kernels()):
-        ld, rd, lb = ctx.kernel_timeline(k)
-        if ld:
-            tl[P.kernel_name(k)[5:]] = [round(lb / 1e3), round(ld / 1e3), round(rd / 1e3)]
-    # hot (L2-warm) for the ratio, same process
-    for _ in range(10):
-        ctx.infer(s)
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(50):
-        ctx.infer(s)
-    e1.record()
-    torch.cuda.synchronize()
-    st2 = ctx.stats()
-    hot_issue = (st2["issue_ns"] - st["issue_ns"]) / 1e3 / max(1, st2["launches"] - st["launches"])
-    print(json.dumps({"hot_issue_us_per_launch": hot_issue,
-                      "cold_issue_us_per_launch": st["issue_ns"] / 1e3 / max(1, st["launches"]),
-                      "cold_us": st["cold_wall_ns"] / 1e3, "cold_py_us": (t1 - t0) / 1e3, "hot_us": 1e3 * e0.elapsed_time(e1) / 50,
-                      "kernels_loaded": st["kernels_loaded"], "code_objects": st["code_objects_loaded"],
-                      "load_us": st["load_ns"] / 1e3, "load_exposed_us": st["load_exposed_ns"] / 1e3,
-                      "issue_us": st["issue_ns"] / 1e3, "gpu_span_us": st["gpu_span_ns"] / 1e3,
-                      "plan_us": st["plan_ns"] / 1e3, "encode_us": st["encode_ns"] / 1e3,
-                      "t_load_done_us": st["load_done_ns"] / 1e3, "t_infer_entry_us": st["infer_entry_ns"] / 1e3,
-                      "t_first_launch_us": st["first_launch_ns"] / 1e3,
-                      "t_last_launch_us": st["last_launch_ns"] / 1e3,
-                      "t_encode_begin_us": st["encode_begin_ns"] / 1e3,
-                      "t_encode_end_us": st["encode_end_ns"] / 1e3,
-                      "timeline": tl}))
-    ctx.close()
+    if path is None:
+        path = os.path.join(tempfile.gettempdir(), f"pask_{model}_b{batch}_{os.getpid()}.pmodel")
+    DeviceModel(spec, alloc=False).save_image(path, x)
+    return path
+
+
+def run_child(image: str, cfg: dict, device: int = 0, hot: int = 0, dump: str | None = None,
+              flush_mb: int = 256, timeout: float = 120.0, env: dict | None = None) -> dict:
+    cmd = [EXE, image, "--cfg", cfg_arg(cfg), "--device", str(device)]
+    if hot:
+        cmd += ["--hot", str(hot), "--flush-mb", str(flush_mb)]
+    if dump:
+        cmd += ["--dump", dump]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout,
+                       env={**os.environ, **(env or {})})
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    if r.returncode != 0 or not lines:
+        raise RuntimeError(f"pask_cold failed (rc {r.returncode}): {r.stderr[-2000:]}")
+    return json.loads(lines[-1])
+
+
+def pctl(vals, q):
+    s = sorted(vals)
+    return s[min(len(s) - 1, int(q * len(s)))]
+
+
+def sample(image: str, cfg: dict, n: int, device: int = 0) -> list[dict]:
+    return [run_child(image, cfg, device) for _ in range(n)]
+
+
+def summarize(samples: list[dict]) -> dict:
+    cold = [s["cold_us"] for s in samples]
+    return {"median_us": statistics.median(cold), "p90_us": pctl(cold, 0.9), "min_us": min(cold),
+            "n": len(cold), "kernels_loaded": samples[0]["kernels_loaded"]}
+
+
+def breakdown(samples: list[dict]) -> dict:
+    """Partition of the cold wall (Fig. 1(b) / Fig. 7 categories, reading G1:
+    loading / issue / GPU execution / other) from timeline = 1 samples, per
+    sample then median:
+      plan       pask_load_model entry -> plan done (parse + Algorithm 1)
+      load       plan done -> every planned kernel uploaded (encode overlaps it)
+      issue      uploads done -> first launch issued (infer entry, first launch)
+      gpu_busy   union of the kernels' [start, end] intervals (timeline stamps)
+      gpu_idle   first launch -> last kernel end, minus busy (issue-paced gaps)
+      other      the rest of the window (sync return)
+    and GPU utilisation = gpu_busy / cold wall (Fig. 6(b))."""
+    rows = []
+    for s in samples:
+        cold = s["cold_us"]
+        plan = s["plan_us"]
+        load = max(0.0, s["t_load_done_us"] - plan)
+        issue = max(0.0, s["t_first_launch_us"] - s["t_load_done_us"])
+        span = s["gpu_span_us"]
+        busy = min(s["gpu_busy_us"], span)
+        other = cold - plan - load - issue - span
+        rows.append({"plan": plan, "load": load, "issue": issue, "gpu_busy": busy, "gpu_idle": span - busy,
+                     "other": other, "cold": cold, "util": busy / cold if cold else 0.0})
+    return {k: round(statistics.median(r[k] for r in rows), 1 if k != "util" else 4) for k in rows[0]}
+
+
+def replicas(image: str, cfg: dict, n_procs: int, trials: int, devices=None, dump_dir: str | None = None,
+             timeout: float = 120.0) -> list[list[dict]]:
+    """trials x n_procs cold starts; in each trial the n_procs children are
+    released into the cold window together (devices[i] per child, default all
+    on device 0: loader contention on one GPU's driver and host)."""
+    devices = devices or [0] * n_procs
+    out = []
+    for t in range(trials):
+        procs = []
+        for i in range(n_procs):
+            cmd = [EXE, image, "--cfg", cfg_arg(cfg), "--device", str(devices[i]), "--wait"]
+            if dump_dir and t == 0:
+                cmd += ["--dump", os.path.join(dump_dir, f"replica{i}.bin")]
+            procs.append(subprocess.Popen(cmd, stdin=subprocess.PIPE, stdout=subprocess.PIPE,
+                                          stderr=subprocess.PIPE, text=True))
+        for p in procs:  # every child set up and waiting
+            line = p.stdout.readline()
+            if line.strip() != "ready":
+                raise RuntimeError(f"replica did not get ready: {line!r} {p.stderr.read()[-2000:]}")
+        for p in procs:  # release them together
+            p.stdin.write("go\n")
+            p.stdin.flush()
+        res = []
+        for p in procs:
+            so, se = p.communicate(timeout=timeout)
+            lines = [l for l in so.splitlines() if l.startswith("{")]
+            if p.returncode != 0 or not lines:
+                raise RuntimeError(f"replica failed (rc {p.returncode}): {se[-2000:]}")
+            res.append(json.loads(lines[-1]))
+        out.append(res)
+    return out
 
 
 def main():
@@ -102,43 +155,35 @@ def main():
     ap.add_argument("--model", default="resnet50")
     ap.add_argument("--n", type=int, default=20)
     ap.add_argument("--schemes", default=",".join(SCHEMES))
-    ap.add_argument("--child", default=None)
     ap.add_argument("--batch", type=int, default=1)
+    ap.add_argument("--hot", type=int, default=200, help="hot inferences of one extra child per scheme")
     a = ap.parse_args()
-    if a.child:
-        child(a.model, a.child, a.batch)
-        return
+    image = write_image(a.model, batch=a.batch)
     out = {}
-    for scheme in a.schemes.split(","):
-        samples = []
-        for _ in range(a.n):
-            r = subprocess.run([sys.executable, __file__, "--model", a.model, "--child", scheme,
-                                "--batch", str(a.batch)],
-                               capture_output=True, text=True, timeout=300,
-                               env={**os.environ, **SCHEME_ENV.get(scheme, {})})
-            line = [l for l in r.stdout.splitlines() if l.startswith("{")]
-            if not line:
-                print(r.stderr[-2000:], file=sys.stderr)
-                continue
-            samples.append(json.loads(line[-1]))
-        if not samples:
-            continue
-        print(f"   {scheme} first-sample timeline [lib, load, ready_at] us: {samples[0]['timeline']}",
-              flush=True)
-        med = {k: statistics.median(s[k] for s in samples) for k in samples[0] if k != "timeline"}
-        cold = sorted(s["cold_us"] for s in samples)
-        med["cold_p90_us"] = cold[min(len(cold) - 1, int(0.9 * len(cold)))]
-        med["cold_over_hot"] = med["cold_us"] / med["hot_us"]
-        med["n"] = len(samples)
-        out[scheme] = med
-        print(f"{a.model:12s} {scheme:18s} cold med {med['cold_us']:8.1f} p90 {med['cold_p90_us']:8.1f} us"
-              f"  hot {med['hot_us']:7.1f}  ratio {med['cold_over_hot']:5.2f}  kernels {med['kernels_loaded']:.0f}"
-              f"  load {med['load_us']:6.1f} exposed {med['load_exposed_us']:6.1f} issue {med['issue_us']:6.1f}"
-              f" gpu {med['gpu_span_us']:6.1f} issue/launch cold {med['cold_issue_us_per_launch']:4.2f}"
-              f" hot {med['hot_issue_us_per_launch']:4.2f} | t: loads {med['t_load_done_us']:6.1f} infer {med['t_infer_entry_us']:6.1f}"
-              f" first {med['t_first_launch_us']:6.1f} last {med['t_last_launch_us']:6.1f}"
-              f" encode [{med['t_encode_begin_us']:6.1f}, {med['t_encode_end_us']:6.1f}]", flush=True)
-    print(json.dumps({"model": a.model, "schemes": out}))
+    try:
+        for scheme in a.schemes.split(","):
+            cfg = SCHEMES[scheme]
+            samples = sample(image, cfg, a.n)
+            tl = sample(image, {**cfg, "timeline": 1}, max(5, a.n // 2))
+            hot = run_child(image, cfg, hot=a.hot) if a.hot else None
+            med = summarize(samples)
+            med["breakdown_us"] = breakdown(tl)
+            med["hot_direct_us"] = hot["hot_median_us"] if hot else None
+            med["cold_over_hot_direct"] = med["median_us"] / hot["hot_median_us"] if hot else None
+            med["queries"], med["hits"], med["lookups"] = (samples[0]["queries"], samples[0]["hits"],
+                                                          samples[0]["lookups"])
+            med["timeline"] = samples[0]["timeline"]
+            out[scheme] = med
+            bd = med["breakdown_us"]
+            print(f"{a.model:12s} {scheme:22s} cold med {med['median_us']:8.1f} p90 {med['p90_us']:8.1f} us"
+                  f" (n {med['n']})  hot(direct) {med['hot_direct_us'] or 0:7.1f}  ratio "
+                  f"{med['cold_over_hot_direct'] or 0:5.2f}  kernels {med['kernels_loaded']:.0f}  "
+                  f"q/h/l {med['queries']:.0f}/{med['hits']:.0f}/{med['lookups']:.0f} | plan {bd['plan']} "
+                  f"load {bd['load']} issue {bd['issue']} busy {bd['gpu_busy']} idle {bd['gpu_idle']} "
+                  f"other {bd['other']} util {bd['util']}", flush=True)
+    finally:
+        os.unlink(image)
+    print(json.dumps({"model": a.model, "batch": a.batch, "schemes": out}))
 
 
 if __name__ == "__main__":

@@ -65,12 +65,28 @@ def test_conv_cases(case):
     _check_spec(conv_spec(c, k, hw, r, s, p, d, act, res))
 
 
-@pytest.mark.parametrize("case", [CONV_CASES[i] for i in (0, 2, 3, 9, 10)], ids=str)
-def test_conv_gather_fallback(case, monkeypatch):
+_GATHER_CHILD = r"""
+import sys
+sys.path.insert(0, sys.argv[1])
+from tests.test_gpu_kernels import CONV_CASES, _check_spec, conv_spec
+for i in (0, 2, 3, 9, 10):
+    _check_spec(conv_spec(*CONV_CASES[i]))
+print("gather ok")
+"""
+
+
+def test_conv_gather_fallback():
     """The cp.async implicit-im2col gather, forced for every non-plain conv with
-    PASK_NO_IM2COL (the 64-channel TMA im2col cases then take it too)."""
-    monkeypatch.setenv("PASK_NO_IM2COL", "1")
-    _check_spec(conv_spec(*case))
+    PASK_NO_IM2COL (the 64-channel TMA im2col cases then take it too).  The
+    runtime reads its switches once per process (tuning.h), so the cases run in
+    a child process started with the switch set."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _GATHER_CHILD, root], env={**os.environ, "PASK_NO_IM2COL": "1"},
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and "gather ok" in r.stdout, r.stderr[-3000:]
 
 
 @pytest.mark.parametrize("s,hw", [(1, 56), (2, 56), (1, 7), (2, 15)])
@@ -127,6 +143,9 @@ def linear_spec(m, kin, nout, act="none", res=False, rows=None, seed=4):
     (128, 768, 3072, "gelu", False, None),  # FFN1 + GELU
     (128, 768, 768, "tanh", False, 1),      # pooler: first row only
     (200, 96, 40, "relu", True, None),      # ragged M, bn 48
+    (8, 8192, 64, "relu", True, None),      # 16-CTA split-K cluster (M <= 64, 128 k-blocks),
+                                            # N % 16 == 0: direct epilogue with residual, rows_per 8
+    (64, 16384, 32, "none", True, None),    # 16-way split, a full 64-row A box, residual
 ])
 def test_linear_cases(m, kin, nout, act, res, rows):
     _check_spec(linear_spec(m, kin, nout, act, res, rows))
