@@ -335,6 +335,8 @@ def main():
                     help="fresh-process cold starts per config (native pask_cold children)")
     ap.add_argument("--timeline-samples", type=int, default=10,
                     help="fresh-process cold starts with cfg.timeline (breakdown, GPU utilisation)")
+    ap.add_argument("--py-cold-samples", type=int, default=5,
+                    help="main config: cold starts in fresh PyTorch processes (framework process state)")
     ap.add_argument("--no-configs", action="store_true",
                     help="skip the other configs' compact block (C1-C4 headline)")
     ap.add_argument("--replica-trials", type=int, default=10, help="N > 1: concurrent cold-start trials")
@@ -627,13 +629,21 @@ def main():
             main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
             nopf = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1}, args.cold_samples))
             main_cold["cold_no_prefault"] = nopf
+            nopr = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1}, args.cold_samples))
+            main_cold["cold_no_prime"] = nopr
+            py = [cs.run_py_child(args.model, cfg, args.batch) for _ in range(args.py_cold_samples)]
+            main_cold["cold_python_process"] = cs.summarize(py) if py else None
         finally:
             os.unlink(image)
         c = main_cold["cold"]
         headline[args.model] = headline_entry(
             c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"], hot_max, direct_max, main_cold["breakdown"],
             c["kernels_loaded"], main_cold["launches"],
-            {"nopf_ms": [round(nopf["median_us"] / 1e3, 3), round(nopf["p90_us"] / 1e3, 3)]})
+            {"nopf_ms": [round(nopf["median_us"] / 1e3, 3), round(nopf["p90_us"] / 1e3, 3)],
+             "noprime_ms": [round(nopr["median_us"] / 1e3, 3), round(nopr["p90_us"] / 1e3, 3)],
+             "py_ms": ([round(main_cold["cold_python_process"]["median_us"] / 1e3, 3),
+                        round(main_cold["cold_python_process"]["p90_us"] / 1e3, 3),
+                        main_cold["cold_python_process"]["n"]] if py else None)})
         if not args.no_configs and args.batch == 1:
             for m in CONFIG_MODELS:
                 if m == args.model:
@@ -711,8 +721,9 @@ def main():
     if replicas:
         line["replicas"] = replicas
     if headline:
-        line["headline"] = {"legend": {"cold_ms": "med,p90,n", "hot_ms": "graph,direct", "cold/hot": "graph,direct",
-                                       "util": "busy/cold", "bd_us": "/".join(BREAKDOWN_KEYS)},
+        line["headline"] = {"legend": {"cold_ms": "med,p90,n (native procs)", "hot_ms": "graph,direct",
+                                       "cold/hot": "graph,direct", "util": "busy/cold",
+                                       "bd_us": "/".join(BREAKDOWN_KEYS), "py_ms": "PyTorch procs"},
                             **headline}
     print(json.dumps(line), flush=True)
     if dist:

@@ -233,6 +233,11 @@ typedef struct {
                          objects, so the first library parse inside the cold window also pays
                          the page faults of reading the image (the Baseline's ELF read,
                          PAPER.md:29); 0 (default) = prefault at create (D8)        */
+  int32_t no_prime;   /* 1 = pask_create does not prime the driver; 0 (default) = it loads,
+                         launches once and unloads a trivial kernel of its own (not a catalog
+                         solution), so the context's one-time module-loader / launch state
+                         exists before the first model load, as in any framework process that
+                         has already run a kernel (D11)                            */
 } pask_config;
 
 typedef enum { PASK_HOW_DIRECT = 0, PASK_HOW_REUSED = 1, PASK_HOW_LOADED = 2 } pask_how;
@@ -280,6 +285,8 @@ typedef struct {
   int32_t max_cluster;         /* largest split-K cluster this device can co-schedule
                                   (cuOccupancyMaxActiveClusters; 16 or 8)           */
   int32_t reserved0;
+  uint64_t prime_ns;           /* pask_create's driver primer (outside the cold
+                                  window; 0 with no_prime)                          */
 } pask_stats_t;
 
 /* Library version (PASK_VERSION). */

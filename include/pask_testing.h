@@ -47,8 +47,15 @@ int32_t pask_test_fake_log(int32_t *out, int32_t *kinds, int32_t cap);
  *                                  (default 0); returns 0
  *   PASK_FAKE_MAX_CLUSTER_LAUNCHED returns the largest cluster size (z) launched
  *                                  since the last reset; value ignored
+ *   PASK_FAKE_PRIMER_LOADS         returns how many times pask_create's driver
+ *                                  primer was uploaded (it is not logged)
  * Unknown knob: -1. */
-enum { PASK_FAKE_OCCUPANCY = 1, PASK_FAKE_CURRENT_DEVICE = 2, PASK_FAKE_MAX_CLUSTER_LAUNCHED = 3 };
+enum {
+  PASK_FAKE_OCCUPANCY = 1,
+  PASK_FAKE_CURRENT_DEVICE = 2,
+  PASK_FAKE_MAX_CLUSTER_LAUNCHED = 3,
+  PASK_FAKE_PRIMER_LOADS = 4
+};
 int32_t pask_test_fake_knob(int32_t knob, int32_t value);
 
 #ifdef __cplusplus

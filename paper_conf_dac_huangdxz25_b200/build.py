@@ -21,7 +21,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 KERNEL_SRC = [os.path.join(CSRC, "kernels", f) for f in
               ("pask_kernels.cu", "conv_gemm.cuh", "attention.cuh", "elementwise.cuh", "ptx.cuh",
-               "pask_params.h")]
+               "pask_params.h", "primer.cuh")]
 HOST_SRC = [os.path.join(CSRC, "runtime", f) for f in ("pask.cpp", "plan.cpp", "driver.cpp")]
 # the fake CUDA driver (include/pask_testing.h) is compiled only into the
 # test-only library libpask_testing.so, never into the product libpask.so
@@ -67,7 +67,8 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # table is generated into _build/spec_catalog.h as PASK_FAMILY_VARIANTS).
 FAMILY_VARIANTS = {"pask_families_tf": 0x30, "pask_families_dwg": 0x1b, "pask_families_cnn": 0x1d,
                    "pask_families_dw": 0x1f, "pask_families": 0x3f}
-EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"]}
+EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"],
+                 "pask_primer": ["pask_primer"]}   # pask_create's driver primer (not a solution)
 EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}"] for k, m in FAMILY_VARIANTS.items()}
 
 # The "tuned library": one specialised conv solution per distinct
@@ -109,7 +110,7 @@ def _gen_spec_sources():
     host += ["#define PASK_SPEC_IMAGES(X) \\"] + [f"  X({spec_name(sp)}) \\" for sp in SPECS] + [""]
     host += ["// packaging 2 families variants (name, memory-case mask), smallest first",
              "#define PASK_FAMILY_VARIANTS(X) \\"] + \
-        [f"  X({k}, {m:#x}) \\" for k, m in FAMILY_VARIANTS.items()] + [""]
+        [f"  X({k}, {m:#x}) \\" for k, m in FAMILY_VARIANTS.items()] + ["", ""]
     for path, text in ((os.path.join(BUILD, "spec_kernels.inc"), "".join(ker)),
                        (os.path.join(BUILD, "spec_catalog.h"), "\n".join(host))):
         old = open(path).read() if os.path.exists(path) else None

@@ -6,6 +6,7 @@
 #include "conv_gemm.cuh"
 #include "attention.cuh"
 #include "elementwise.cuh"
+#include "primer.cuh"
 
 using namespace pask;
 
@@ -149,6 +150,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1) pask_all(const __grid_constan
     mem_dispatch(p.m);
   }
 }
+#endif
+
+#if defined(PASK_ONLY_KERNEL) && PASK_ONLY_KERNEL_pask_primer  // own code object only
+// Not a solution: pask_create's driver primer (primer.cuh, D11).
+__global__ void __launch_bounds__(128, 1) pask_primer(const __grid_constant__ PrimerParams p) { primer_body(p); }
 #endif
 
 // Per-problem specialised conv solutions (the tuned library of the Baseline

@@ -152,6 +152,14 @@ struct alignas(16) MemParams {
   int32_t kind;  // MemKind
 };
 
+// pask_create's driver primer (primer.cuh; not a solution, D11).
+struct alignas(64) PrimerParams {
+  CUtensorMap tmap_a;  // 3-D {64, 128, 1} bf16, SWIZZLE_128B
+  CUtensorMap tmap_b;  // 3-D {64, 64, 1} bf16, SWIZZLE_128B
+  float* out;          // [128][64] fp32
+  int32_t run;         // 0: return at once (how pask_create launches it)
+};
+
 // Single-function entry (pask_config.packaging = 3): the contraction body and the
 // memory-bound family in ONE CUfunction, `pask_all`, so a model's whole catalog
 // becomes resident with one code upload.  g.family 0 runs g, 1 runs m (m lies at

@@ -28,12 +28,15 @@ std::vector<int32_t> g_ids, g_kinds;
 bool g_loaded[PASK_MAX_KERNELS] = {};
 constexpr int32_t kFakeMemFamilyId = PASK_MAX_KERNELS - 1;  // id logged for the `pask_mem` entry
 constexpr int32_t kFakeAllId = PASK_MAX_KERNELS - 2;        // id logged for the `pask_all` entry
+constexpr int32_t kFakePrimerId = PASK_MAX_KERNELS - 3;     // pask_create's primer: never logged
+std::atomic<int32_t> g_primer_loads{0};
 
 int32_t kernel_of_name(const char* name) {
   for (int32_t k = 0; k < num_kernels(); ++k)
     if (strcmp(catalog(k).name, name) == 0) return k;
   if (strcmp(name, "pask_mem") == 0) return kFakeMemFamilyId;  // packaging-2 family entry
   if (strcmp(name, "pask_all") == 0) return kFakeAllId;        // packaging-3 single entry
+  if (strcmp(name, "pask_primer") == 0) return kFakePrimerId;  // driver primer (pask_create)
   return -1;
 }
 void sleep_us(int us) {
@@ -126,6 +129,10 @@ CUresult f_kernel_get_fn(CUfunction* f, CUkernel k) {
 }
 CUresult f_func_load(CUfunction f) {
   const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
+  if (id == kFakePrimerId) {
+    g_primer_loads.fetch_add(1);
+    return CUDA_SUCCESS;
+  }
   {
     std::lock_guard<std::mutex> lk(g_mu);
     if (id >= 0 && id < PASK_MAX_KERNELS) g_loaded[id] = true;
@@ -145,6 +152,7 @@ CUresult f_func_set_attr(CUfunction, CUfunction_attribute, int) { return CUDA_SU
 std::atomic<uintptr_t> g_capture_stream{0};
 CUresult f_launch(const CUlaunchConfig* cfg, CUfunction f, void**, void**) {
   const int32_t id = static_cast<int32_t>(reinterpret_cast<uintptr_t>(f) - kFnBase);
+  if (id == kFakePrimerId) return CUDA_SUCCESS;
   bool loaded;
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -277,6 +285,7 @@ PASK_API int pask_test_fake_driver(int32_t enable, int32_t load_us, int32_t fail
   g_current.store(0x10);
   g_occupancy.store(1);
   g_max_cluster_z.store(0);
+  g_primer_loads.store(0);
   if (enable) {
     g_fake = make_fake();
     driver_override(&g_fake);
@@ -292,6 +301,7 @@ PASK_API int32_t pask_test_fake_knob(int32_t knob, int32_t value) {
     case PASK_FAKE_OCCUPANCY: g_occupancy.store(value); return 0;
     case PASK_FAKE_CURRENT_DEVICE: g_current.store(0x10 + static_cast<uintptr_t>(value)); return 0;
     case PASK_FAKE_MAX_CLUSTER_LAUNCHED: return g_max_cluster_z.load();
+    case PASK_FAKE_PRIMER_LOADS: return g_primer_loads.load();
     default: return -1;
   }
 }

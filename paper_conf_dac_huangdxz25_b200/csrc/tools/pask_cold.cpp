@@ -21,6 +21,7 @@
 // No PyTorch, no Python: the whole process is native, so a sample costs
 // milliseconds of process start instead of seconds of interpreter start.
 #include <dlfcn.h>
+#include <malloc.h>
 #include <stdint.h>
 #include <stdio.h>
 #include <stdlib.h>
@@ -29,6 +30,8 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <atomic>
+#include <thread>
 #include <chrono>
 #include <string>
 #include <type_traits>
@@ -171,7 +174,7 @@ void set_cfg(pask_config* c, const std::string& kv) {
 #define F(name) \
   if (k == #name) { c->name = v; return; }
   F(reuse) F(search) F(milestone) F(proactive) F(pdl) F(instrument) F(packaging) F(interleave) F(graph)
-  F(catalog) F(branches) F(timeline) F(no_prefault)
+  F(catalog) F(branches) F(timeline) F(no_prefault) F(no_prime)
 #undef F
   die("unknown pask_config field " + k);
 }
@@ -193,11 +196,12 @@ int main(int argc, char** argv) {
     return 1;
   }
   const char* model = argv[1];
-  pask_config cfg{1, 0, 0, 2, 1, 0, 0, 0, 0, 0, 0, 0, 0};  // the library defaults (pask.h)
-  int device = 0, hot = 0, flush_mb = 256;
-  bool wait = false, plan_only = false;
-  double sleep_ms = 50;
+  pask_config cfg{1, 0, 0, 2, 1, 0, 0, 0, 0, 0, 0, 0, 0, 0};  // the library defaults (pask.h)
+  int device = 0, hot = 0, flush_mb = 256, warm_heap_mb = 0;
+  bool wait = false, plan_only = false, bg_spin = false, cudart = false;
+  double sleep_ms = 50, spin_ms = 0;
   const char* dump = nullptr;
+  std::string pre_image;  // experiment: PATH:function loaded, uploaded and unloaded before pask_create
   for (int i = 2; i < argc; ++i) {
     const std::string a = argv[i];
     auto next = [&]() -> const char* {
@@ -222,6 +226,17 @@ int main(int argc, char** argv) {
       plan_only = true;
     } else if (a == "--sleep-ms") {
       sleep_ms = atof(next());
+    } else if (a == "--warm-heap-mb") {  // experiment: a warm malloc arena, as in a long-lived server
+      warm_heap_mb = atoi(next());
+    } else if (a == "--pre-image") {
+      pre_image = next();
+    } else if (a == "--cudart") {  // experiment: initialise the CUDA runtime first, as a framework does
+      cudart = true;
+    } else if (a == "--bg-spin") {  // experiment: a second thread busy through the cold window
+      bg_spin = true;
+    } else if (a == "--spin-ms") {  // busy-wait (core kept awake) instead of sleeping before t0
+      spin_ms = atof(next());
+      sleep_ms = 0;
     } else if (a == "--hot") {
       hot = atoi(next());
     } else if (a == "--flush-mb") {
@@ -231,6 +246,14 @@ int main(int argc, char** argv) {
     } else {
       die("unknown argument " + a);
     }
+  }
+  if (warm_heap_mb > 0) {
+    mallopt(M_MMAP_THRESHOLD, 512 << 20);
+    mallopt(M_TRIM_THRESHOLD, 1 << 30);
+    mallopt(M_TOP_PAD, 64 << 20);
+    void* h = malloc(static_cast<size_t>(warm_heap_mb) << 20);
+    memset(h, 1, static_cast<size_t>(warm_heap_mb) << 20);
+    free(h);
   }
   Image im = read_image(model);
   if (plan_only) {  // no GPU: check the image round trip through the host planner
@@ -260,6 +283,16 @@ int main(int argc, char** argv) {
   const Cu cu = resolve();
   g_cu = &cu;
   // ---- outside the cold window: context, memory, weights, input
+  if (cudart) {
+    void* rt = dlopen("libcudart.so.12", RTLD_NOW | RTLD_GLOBAL);
+    if (!rt) die("libcudart.so.12 not found");
+    using FreeFn = int (*)(void*);
+    using MallocFn = int (*)(void**, size_t);
+    auto cfree = reinterpret_cast<FreeFn>(dlsym(rt, "cudaFree"));
+    auto cmalloc = reinterpret_cast<MallocFn>(dlsym(rt, "cudaMalloc"));
+    void* p0 = nullptr;
+    if (!cfree || !cmalloc || cfree(nullptr) != 0 || cmalloc(&p0, 1 << 21) != 0) die("cudart init failed");
+  }
   ck(cu.init(0), "cuInit");
   CUdevice dev;
   ck(cu.device_get(&dev, device), "cuDeviceGet");
@@ -316,6 +349,38 @@ int main(int argc, char** argv) {
   g.outputs = im.outputs.data();
   g.workspace = im.ws_bytes ? reinterpret_cast<void*>(base + ws_off) : nullptr;
   g.workspace_bytes = im.ws_bytes;
+  std::atomic<bool> bg_stop{false};
+  std::thread bg;
+  if (bg_spin)
+    bg = std::thread([&] {
+      volatile uint64_t x = 0;
+      while (!bg_stop.load(std::memory_order_relaxed)) x = x + 1;
+    });
+  if (!pre_image.empty()) {
+    const size_t colon = pre_image.rfind(':');
+    const std::string path = pre_image.substr(0, colon), fn = pre_image.substr(colon + 1);
+    FILE* f = fopen(path.c_str(), "rb");
+    if (!f) die("cannot open " + path);
+    std::vector<unsigned char> img;
+    unsigned char buf[65536];
+    size_t nrd;
+    while ((nrd = fread(buf, 1, sizeof buf, f)) > 0) img.insert(img.end(), buf, buf + nrd);
+    fclose(f);
+    void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_LOCAL);
+    auto lload = reinterpret_cast<decltype(&::cuLibraryLoadData)>(dlsym(h, "cuLibraryLoadData"));
+    auto lget = reinterpret_cast<decltype(&::cuLibraryGetKernel)>(dlsym(h, "cuLibraryGetKernel"));
+    auto kfn = reinterpret_cast<decltype(&::cuKernelGetFunction)>(dlsym(h, "cuKernelGetFunction"));
+    auto fload = reinterpret_cast<decltype(&::cuFuncLoad)>(dlsym(h, "cuFuncLoad"));
+    auto lunload = reinterpret_cast<decltype(&::cuLibraryUnload)>(dlsym(h, "cuLibraryUnload"));
+    CUlibrary lib;
+    CUkernel k;
+    CUfunction fnc;
+    ck(lload(&lib, img.data(), nullptr, nullptr, 0, nullptr, nullptr, 0), "pre-image load");
+    ck(lget(&k, lib, fn.c_str()), "pre-image kernel");
+    ck(kfn(&fnc, k), "pre-image function");
+    ck(fload(fnc), "pre-image upload");
+    ck(lunload(lib), "pre-image unload");
+  }
   pask_ctx* pc = nullptr;
   pk(pask_create(&pc, device, &cfg), "pask_create");
   const uint64_t t_ready = now_ns();
@@ -326,6 +391,11 @@ int main(int argc, char** argv) {
     if (!fgets(line, sizeof line, stdin)) die("stdin closed before go");
   }
   if (sleep_ms > 0) usleep(static_cast<useconds_t>(sleep_ms * 1000));  // idle before the window
+  if (spin_ms > 0) {
+    const uint64_t until = now_ns() + static_cast<uint64_t>(spin_ms * 1e6);
+    while (now_ns() < until) {
+    }
+  }
   ck(cu.ctx_sync(), "cuCtxSynchronize");
   // ---- the cold window: pask_load_model entry -> first inference complete
   const uint64_t t0 = now_ns();
@@ -334,6 +404,8 @@ int main(int argc, char** argv) {
   pk(pask_infer(pc, nullptr, nullptr, nullptr), "pask_infer");
   pk(pask_sync(pc), "pask_sync");
   const uint64_t t1 = now_ns();
+  bg_stop.store(true);
+  if (bg.joinable()) bg.join();
   pask_stats_t st;
   pk(pask_stats(pc, &st), "pask_stats");
   std::string js = "{";
@@ -368,6 +440,7 @@ int main(int argc, char** argv) {
   kv("t_encode_end_us", st.encode_end_ns / 1e3);
   kv("launches", static_cast<double>(st.launches));
   kv("prefault_us", st.prefault_ns / 1e3);
+  kv("prime_us", st.prime_ns / 1e3);
   kv("max_cluster", st.max_cluster);
   {  // per-kernel load timeline [lib_us, load_us, ready_at_us]
     js += "\"timeline\": {";

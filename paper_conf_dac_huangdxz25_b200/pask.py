@@ -13,7 +13,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libpask.so")
 # test-only build of the same library plus the fake CUDA driver of
 # include/pask_testing.h (never loaded by the product path)
-TESTING_LIB_PATH = os.path.join(_PKG, "libpask_testing.so")
+TESTING_LIB_PATH = os.environ.get("PASK_TESTING_LIB", os.path.join(_PKG, "libpask_testing.so"))
 
 # ---------------------------------------------------------------- enums (pask.h)
 OK, EINVAL, EUNSUPPORTED, ECUDA, ENOMEM, ESTATE = 0, -1, -2, -3, -4, -5
@@ -61,7 +61,7 @@ class Config(C.Structure):
                 ("proactive", C.c_int32), ("pdl", C.c_int32), ("instrument", C.c_int32),
                 ("packaging", C.c_int32), ("interleave", C.c_int32), ("graph", C.c_int32),
                 ("catalog", C.c_int32), ("branches", C.c_int32), ("timeline", C.c_int32),
-                ("no_prefault", C.c_int32)]
+                ("no_prefault", C.c_int32), ("no_prime", C.c_int32)]
 
 
 class Binding(C.Structure):
@@ -80,7 +80,8 @@ class Stats(C.Structure):
                 ("first_launch_ns", C.c_uint64), ("last_launch_ns", C.c_uint64),
                 ("encode_begin_ns", C.c_uint64), ("encode_end_ns", C.c_uint64),
                 ("kernel_span_ns", C.c_uint64), ("prefault_ns", C.c_uint64),
-                ("prefault_bytes", C.c_uint64), ("max_cluster", C.c_int32), ("reserved0", C.c_int32)]
+                ("prefault_bytes", C.c_uint64), ("max_cluster", C.c_int32), ("reserved0", C.c_int32),
+                ("prime_ns", C.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -92,7 +93,7 @@ EXPORTS = ["pask_version", "pask_create", "pask_plan", "pask_workspace_bytes", "
            "pask_kernel_function",
            "pask_kernel_timeline", "pask_node_times", "pask_node_intervals", "pask_promote"]
 TEST_EXPORTS = ["pask_test_fake_driver", "pask_test_fake_log", "pask_test_fake_knob"]   # pask_testing.h
-FAKE_OCCUPANCY, FAKE_CURRENT_DEVICE, FAKE_MAX_CLUSTER_LAUNCHED = 1, 2, 3
+FAKE_OCCUPANCY, FAKE_CURRENT_DEVICE, FAKE_MAX_CLUSTER_LAUNCHED, FAKE_PRIMER_LOADS = 1, 2, 3, 4
 
 _libs = {}
 _use_testing = False
@@ -172,9 +173,9 @@ def function_name(k, packaging):
 
 
 def config(reuse=1, search=0, milestone=0, proactive=2, pdl=1, instrument=0, packaging=0,
-           interleave=0, graph=0, catalog=0, branches=0, timeline=0, no_prefault=0):
+           interleave=0, graph=0, catalog=0, branches=0, timeline=0, no_prefault=0, no_prime=0):
     return Config(reuse, search, milestone, proactive, pdl, instrument, packaging, interleave, graph,
-                  catalog, branches, timeline, no_prefault)
+                  catalog, branches, timeline, no_prefault, no_prime)
 
 
 def test_fake_driver(enable=True, load_us=0, fail_kernel=-1):

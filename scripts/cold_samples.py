@@ -77,6 +77,43 @@ def run_child(image: str, cfg: dict, device: int = 0, hot: int = 0, dump: str | 
     return json.loads(lines[-1])
 
 
+def py_child(model: str, cfg: dict, batch: int = 1):
+    """A cold start in a fresh PyTorch process (the framework process a model
+    server runs in): torch allocates and uploads, pask_create, 50 ms idle, then
+    the cold window.  Prints the same keys as the native sampler."""
+    import time
+
+    import torch
+
+    from paper_conf_dac_huangdxz25_b200 import pask as P
+    from paper_conf_dac_huangdxz25_b200.model import DeviceModel
+    from workloads import build_model
+    spec, x = build_model(model, **({"batch": batch} if batch != 1 else {}))
+    dm = DeviceModel(spec)
+    dm.set_input(x)
+    torch.cuda.synchronize()
+    ctx = P.Context(0, P.config(**cfg))
+    s = torch.cuda.current_stream().cuda_stream
+    time.sleep(0.05)
+    torch.cuda.synchronize()
+    ctx.load_model(dm.graph, plan=False)
+    ctx.infer(s)
+    ctx.sync()
+    st = ctx.stats()
+    print(json.dumps({"cold_us": st["cold_wall_ns"] / 1e3, "kernels_loaded": st["kernels_loaded"],
+                      "t_load_done_us": st["load_done_ns"] / 1e3, "gpu_span_us": st["gpu_span_ns"] / 1e3}))
+    ctx.close()
+
+
+def run_py_child(model: str, cfg: dict, batch: int = 1, timeout: float = 300.0) -> dict:
+    r = subprocess.run([sys.executable, os.path.abspath(__file__), "--py-child", model, "--cfg", cfg_arg(cfg),
+                        "--batch", str(batch)], capture_output=True, text=True, timeout=timeout)
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    if r.returncode != 0 or not lines:
+        raise RuntimeError(f"python cold child failed (rc {r.returncode}): {r.stderr[-2000:]}")
+    return json.loads(lines[-1])
+
+
 def pctl(vals, q):
     s = sorted(vals)
     return s[min(len(s) - 1, int(q * len(s)))]
@@ -157,8 +194,39 @@ def main():
     ap.add_argument("--schemes", default=",".join(SCHEMES))
     ap.add_argument("--batch", type=int, default=1)
     ap.add_argument("--hot", type=int, default=200, help="hot inferences of one extra child per scheme")
+    ap.add_argument("--replicas", default=None,
+                    help="e.g. 1,2,4,8: N processes on ONE GPU released into the cold start together "
+                         "(SURVEY.md §8(e) loader contention), --n trials each")
+    ap.add_argument("--py-child", default=None, help=argparse.SUPPRESS)
+    ap.add_argument("--cfg", default="", help=argparse.SUPPRESS)
     a = ap.parse_args()
+    if a.py_child:
+        py_child(a.py_child, {k: int(v) for k, v in (kv.split("=") for kv in a.cfg.split(",") if kv)}, a.batch)
+        return
     image = write_image(a.model, batch=a.batch)
+    if a.replicas:
+        cfg = SCHEMES["pask_families_branches"]
+        res = {}
+        try:
+            for n in [int(v) for v in a.replicas.split(",")]:
+                trials = replicas(image, cfg, n, a.n)
+                cold = [r["cold_us"] for t in trials for r in t]
+                per = [[round(t[i]["cold_us"], 1) for t in trials] for i in range(n)]
+                res[n] = {"cold_med_us": statistics.median(cold), "cold_p90_us": pctl(cold, 0.9),
+                          "cold_max_us": max(cold), "trials": a.n,
+                          "per_replica_med_us": [round(statistics.median(v), 1) for v in per],
+                          "kernels_loaded": sorted({int(r["kernels_loaded"]) for t in trials for r in t}),
+                          "load_done_med_us": statistics.median(r["t_load_done_us"] for t in trials for r in t)}
+                base = res[min(res)]["cold_med_us"]
+                res[n]["contention"] = res[n]["cold_med_us"] / base
+                print(f"{a.model} replicas {n}: cold med {res[n]['cold_med_us']:7.1f} p90 {res[n]['cold_p90_us']:7.1f} "
+                      f"max {res[n]['cold_max_us']:7.1f} us  contention {res[n]['contention']:.2f}  load_done "
+                      f"{res[n]['load_done_med_us']:6.1f}  kernels {res[n]['kernels_loaded']}  per-replica "
+                      f"{res[n]['per_replica_med_us']}", flush=True)
+        finally:
+            os.unlink(image)
+        print(json.dumps({"model": a.model, "replicas_one_gpu": res}))
+        return
     out = {}
     try:
         for scheme in a.schemes.split(","):

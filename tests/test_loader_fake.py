@@ -362,3 +362,20 @@ def test_timeline_api_states():
         ctx.node_intervals()
     assert ei.value.code == P.ESTATE
     ctx.close()
+
+
+def test_primer_outside_the_plan():
+    """pask_create's driver primer (D11) uploads its own trivial kernel
+    once per context, never a catalog solution, and not with no_prime = 1; the
+    model's loads and launches are unchanged by it."""
+    spec, _ = build_model("tiny_cnn")
+    for no_prime, want in ((0, 1), (1, 0)):
+        P.test_fake_driver(True)
+        ctx = P.Context(0, P.config(no_prime=no_prime))
+        assert P.test_fake_knob(P.FAKE_PRIMER_LOADS) == want
+        plan = ctx.load_model(DeviceModel(spec, alloc=False).graph)
+        ctx.infer(0)
+        ctx.sync()
+        ctx.close()
+        log = P.test_fake_log()
+        assert [k for k, kind in log if kind == 1] == [b[2] for b in plan]
