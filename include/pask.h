@@ -102,7 +102,10 @@ typedef enum {
   PASK_K_LAYERNORM = 8,  /* cat (LAYERNORM, bf16, ROWMAJOR)                             */
   PASK_K_ATTENTION = 9,  /* fused attention, tcgen05/TMEM; cat (ATTENTION, bf16, ROWMAJOR) */
   PASK_K_CONV_IGEMM_PT = 10, /* implicit-GEMM conv as persistent tiles (large M); cat (CONV, bf16, NHWC) */
-  PASK_NUM_KERNELS = 11  /* size of the generic catalog; ids >= 11 are the per-problem
+  PASK_K_GEMV = 11,      /* weight-streaming GEMV for GEMMs of <= 8 rows with a weight operand
+                            [N][K] (FC layers at batch <= 8, BERT's pooler); cat (GEMM, bf16,
+                            ROWMAJOR); D12                                       */
+  PASK_NUM_KERNELS = 12  /* size of the generic catalog; ids >= 12 are the per-problem
                             specialised conv solutions of the tuned catalog (one per
                             (R, S, stride, pad, dilation, C) of configs C1-C3, category
                             (CONV, bf16, NHWC), applicable to exactly that problem

@@ -27,10 +27,14 @@ import math
 LAYOUT, CONV, DWCONV, POOL, GEMM, SOFTMAX, LAYERNORM, ATTENTION = range(8)
 
 # kernel catalog ids
-K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN, K_ATTN, K_IGEMM_PT = range(11)
+K_LAYOUT, K_IGEMM, K_CONV1X1, K_DW, K_POOL, K_GAVG, K_GEMM, K_SOFTMAX, K_LN, K_ATTN, K_IGEMM_PT, K_GEMV = \
+    range(12)
 KERNEL_NAMES = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw",
                 "pask_pool", "pask_pool_gavg", "pask_gemm", "pask_softmax", "pask_layernorm",
-                "pask_attention", "pask_conv_igemm_pt"]
+                "pask_attention", "pask_conv_igemm_pt", "pask_gemv"]
+# s* of a GEMM with at most this many rows (an FC layer at batch <= 8, BERT's
+# pooler) is the weight-streaming GEMV solution (reading D12)
+GEMV_MAX_ROWS = 8
 # s* of a dense conv with more output rows N*P*Q than 148 SMs x 128-row tiles is the
 # persistent-tile implicit-GEMM solution
 PERSISTENT_ROWS = 148 * 128
@@ -44,7 +48,7 @@ SPECS = sorted([
 ] + [(1, 1, 2, 0, 1, c) for c in (256, 512, 1024)]
   + [(3, 3, 1, 1, 1, c) for c in (8, 16, 32, 64, 128, 256, 512)]
   + [(3, 3, 2, 1, 1, c) for c in (8, 128, 256, 512)] + [(7, 7, 2, 3, 1, 8)])
-N_GENERIC = 11
+N_GENERIC = 12
 KERNEL_NAMES = KERNEL_NAMES + ["pask_conv_spec_r%ds%du%dp%dd%dc%d" % sp for sp in SPECS]
 
 # category key (op class, dtype, layout): dtype 0 = bf16 compute path, layouts
@@ -61,6 +65,7 @@ CATEGORY = {
     K_LN: (LAYERNORM, 0, 2),
     K_ATTN: (ATTENTION, 0, 2),
     K_IGEMM_PT: (CONV, 0, 1),
+    K_GEMV: (GEMM, 0, 2),
 }
 CATEGORY.update({N_GENERIC + i: (CONV, 0, 1) for i in range(len(SPECS))})
 
@@ -110,6 +115,11 @@ def is_applicable(kid, p):
         return (op == GEMM and p["gk"] % 8 == 0 and p["lda"] % 8 == 0 and p["ldb"] % 8 == 0
                 and p["off_a"] % 8 == 0 and p["off_b"] % 8 == 0
                 and p["gm"] >= 1 and p["gn"] >= 1 and p["batch"] >= 1)
+    if kid == K_GEMV:   # DESIGN.md D12: weight operand [N][K], one GEMM, few rows
+        return (op == GEMM and p["b_weights"] == 1 and p["trans_b"] == 1 and p["batch"] == 1
+                and 1 <= p["gm"] <= GEMV_MAX_ROWS and p["gn"] >= 1 and p["gk"] % 8 == 0
+                and p["lda"] % 8 == 0 and p["ldb"] % 8 == 0
+                and p["off_a"] % 8 == 0 and p["off_b"] % 8 == 0)
     if kid == K_SOFTMAX:
         return op == SOFTMAX and 1 <= p["cols"] <= 16384
     if kid == K_LN:
@@ -142,7 +152,7 @@ def static_choice(p, catalog="generic"):
     if op == POOL:
         return K_GAVG if (p["global"] == 1 and p["pool_mode"] == 1) else K_POOL
     if op == GEMM:
-        return K_GEMM
+        return K_GEMV if is_applicable(K_GEMV, p) else K_GEMM
     if op == SOFTMAX:
         return K_SOFTMAX
     if op == LAYERNORM:
@@ -154,7 +164,8 @@ def static_choice(p, catalog="generic"):
 
 _ZERO = dict(op=0, n=0, h=0, w=0, c=0, k=0, r=0, s=0, stride_h=0, stride_w=0, pad_h=0,
              pad_w=0, dil_h=0, dil_w=0, groups=0, p=0, q=0, pool_mode=0, **{"global": 0},
-             gm=0, gn=0, gk=0, batch=0, lda=0, ldb=0, off_a=0, off_b=0, rows=0, cols=0)
+             gm=0, gn=0, gk=0, batch=0, lda=0, ldb=0, off_a=0, off_b=0, trans_b=0, b_weights=0,
+             rows=0, cols=0)
 
 
 def problems_from_spec(spec):
@@ -200,18 +211,18 @@ def problems_from_spec(spec):
             if len(shapes[src]) == 4:        # flattened image: K over the device channels
                 _, c, h, w = shapes[src]
                 kin = h * w * devc.get(src, c)
-            p.update(op=GEMM, gm=m, gn=nout, gk=kin, batch=1, lda=kin, ldb=kin)
+            p.update(op=GEMM, gm=m, gn=nout, gk=kin, batch=1, lda=kin, ldb=kin, trans_b=1, b_weights=1)
         elif op == "qk":
             s_, three_h = shapes[layer["inputs"][0]]
             hd = layer["head_dim"]
             p.update(op=GEMM, gm=s_, gn=s_, gk=hd, batch=layer["heads"], lda=three_h,
-                     ldb=three_h, off_a=0, off_b=three_h // 3)
+                     ldb=three_h, off_a=0, off_b=three_h // 3, trans_b=1, b_weights=0)
         elif op == "pv":
             heads, s_, _ = shapes[layer["inputs"][0]]
             three_h = shapes[layer["inputs"][1]][1]
             hd = layer["head_dim"]
             p.update(op=GEMM, gm=s_, gn=hd, gk=s_, batch=heads, lda=s_, ldb=three_h,
-                     off_a=0, off_b=2 * (three_h // 3))
+                     off_a=0, off_b=2 * (three_h // 3), trans_b=0, b_weights=0)
         elif op == "attention":
             s_, three_h = shapes[layer["inputs"][0]]
             p.update(op=ATTENTION, gm=s_, gn=layer["heads"], gk=layer["head_dim"], batch=1,

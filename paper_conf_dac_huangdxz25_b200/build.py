@@ -54,19 +54,19 @@ def _stale(target, deps):
 # catalog order (include/pask.h PASK_K_*)
 KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "pask_pool",
            "pask_pool_gavg", "pask_gemm", "pask_softmax", "pask_layernorm", "pask_attention",
-           "pask_conv_igemm_pt"]
+           "pask_conv_igemm_pt", "pask_gemv"]
 # Extra code objects that are not catalog ids: packaging 2's operator families
 # (D8) -- the generic implicit-GEMM entry and the memory-bound family
 # entry `pask_mem` in ONE code object.  name -> entries compiled into it.
 # The families object comes in variants by the memory cases compiled in
 # (PASK_MEM_MASK, bit per MemKind: layout 0, dw 1, pool 2, gavg 3, softmax 4,
-# LayerNorm 5); the runtime loads the smallest covering the model's solutions
+# LayerNorm 5, GEMV 6); the runtime loads the smallest covering the model's solutions
 # (dwg = depthwise + global pool without the windowed pool: MobileNetV2).
 # Packaging 3 (D10): both families behind the single entry `pask_all`.
 # Smallest first: the runtime takes the first variant covering the plan (the
 # table is generated into _build/spec_catalog.h as PASK_FAMILY_VARIANTS).
-FAMILY_VARIANTS = {"pask_families_tf": 0x30, "pask_families_dwg": 0x1b, "pask_families_cnn": 0x1d,
-                   "pask_families_dw": 0x1f, "pask_families": 0x3f}
+FAMILY_VARIANTS = {"pask_families_tf": 0x70, "pask_families_dwg": 0x5b, "pask_families_cnn": 0x5d,
+                   "pask_families_dw": 0x5f, "pask_families": 0x7f}
 EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"],
                  "pask_primer": ["pask_primer"]}   # pask_create's driver primer (not a solution)
 EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}"] for k, m in FAMILY_VARIANTS.items()}

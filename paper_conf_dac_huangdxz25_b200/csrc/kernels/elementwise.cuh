@@ -478,4 +478,79 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   }
 }
 
+// ---------------------------------------------------------------- K13 GEMV
+// FC layers at batch <= 8 and BERT's pooler (D12): every weight byte
+// is read once, so the layer is one HBM stream of the [N][K] weights.  A lane
+// holds up to kGemvPre 16-byte weight vectors in registers, loaded BEFORE
+// griddepcontrol.wait (weights do not depend on the previous layer), so the HBM
+// round trip overlaps the previous layer's tail; after the wait it reads the M
+// activation rows (L2-resident) and accumulates in fp32.  Lane partials are
+// combined by the fixed xor tree, the K slices of a column in slice order.
+constexpr int kGemvPre = 8;
+__device__ __noinline__ float gemv_act_slow(float v, int act) { return apply_act(v, act); }
+// fp32 dot of two 8 x bf16 vectors added to acc (bf16 -> fp32 is a 16-bit shift)
+__device__ __forceinline__ float dot8(const uint4& a, const uint4& b, float acc) {
+  const uint32_t av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    acc = fmaf(__uint_as_float(av[i] << 16), __uint_as_float(bv[i] << 16), acc);
+    acc = fmaf(__uint_as_float(av[i] & 0xffff0000u), __uint_as_float(bv[i] & 0xffff0000u), acc);
+  }
+  return acc;
+}
+__device__ __forceinline__ void gemv_body(const GemvParams& p) {
+  // [slice][column in CTA][row] partials in the dynamic smem (2 KB, set by the
+  // host): the family entries share one static-smem budget with the contraction
+  extern __shared__ uint8_t smem_raw[];
+  float (*part)[8][8] = reinterpret_cast<float (*)[8][8]>(smem_raw);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nc = 1 << p.nc_log2, slices = (blockDim.x >> 5) >> p.nc_log2;
+  const int cc = warp & (nc - 1), slice = warp >> p.nc_log2;
+  const int n = (blockIdx.x << p.nc_log2) + cc;
+  const int per = p.per;                           // 16-byte vectors per K slice (host)
+  const int v0 = slice * per + lane, v1 = min(p.K >> 3, slice * per + per);
+  const bool live = n < p.N;
+  const uint4* w = reinterpret_cast<const uint4*>(reinterpret_cast<const __nv_bfloat16*>(p.w) +
+                                                  static_cast<int64_t>(live ? n : 0) * p.ldb) + v0;
+  uint4 wv[kGemvPre];
+#pragma unroll
+  for (int j = 0; j < kGemvPre; ++j)
+    wv[j] = (live && v0 + 32 * j < v1) ? __ldg(w + 32 * j) : make_uint4(0, 0, 0, 0);
+  pdl_wait();
+  pdl_launch_dependents();
+  // rows one at a time (compact code: an upload costs ~1.1 us per KB of SASS)
+#pragma unroll 1
+  for (int m = 0; m < p.M; ++m) {
+    const uint4* x = reinterpret_cast<const uint4*>(reinterpret_cast<const __nv_bfloat16*>(p.x) +
+                                                    static_cast<int64_t>(m) * p.lda) + v0;
+    float acc = 0.f;
+    if (live) {
+#pragma unroll
+      for (int j = 0; j < kGemvPre; ++j)
+        if (v0 + 32 * j < v1) acc = dot8(__ldg(x + 32 * j), wv[j], acc);
+#pragma unroll 1
+      for (int j = kGemvPre; v0 + 32 * j < v1; ++j) acc = dot8(__ldg(x + 32 * j), __ldg(w + 32 * j), acc);
+    }
+    acc = warp_sum(acc);
+    if (lane == 0) part[slice][cc][m] = acc;
+  }
+  __syncthreads();
+  const int t = threadIdx.x;
+  if (t < 64) {
+    const int c = t & 7, m = t >> 3;               // column in CTA, row
+    const int col = (blockIdx.x << p.nc_log2) + c;
+    if (c < nc && m < p.M && col < p.N) {
+      float v = 0.f;
+      for (int s = 0; s < slices; ++s) v += part[s][c][m];
+      if (p.bias) v += __ldg(p.bias + col);
+      const int64_t o = static_cast<int64_t>(m) * p.ldc + col;
+      if (p.res) v += __bfloat162float(reinterpret_cast<const __nv_bfloat16*>(p.res)[o]);
+      if (p.act == 1) v = fmaxf(v, 0.f);
+      else if (p.act == 2) v = fminf(fmaxf(v, 0.f), 6.f);
+      else if (p.act >= 3) v = gemv_act_slow(v, p.act);
+      reinterpret_cast<__nv_bfloat16*>(p.y)[o] = __float2bfloat16_rn(v);
+    }
+  }
+}
+
 }  // namespace pask

@@ -18,7 +18,7 @@ static_assert(kTimelineStride == 4096, "TimelineScope (ptx.cuh) hard-codes the e
 // model's bound solutions (D8).  A case compiled out traps: the host
 // never binds it, and if it did the launch fails loudly instead of writing nothing.
 #ifndef PASK_MEM_MASK
-#define PASK_MEM_MASK 0x3f
+#define PASK_MEM_MASK 0x7f
 #endif
 #define PASK_MEM_CASE(k, body) \
   case k:                     \
@@ -34,6 +34,7 @@ __device__ __forceinline__ void mem_dispatch(const MemParams& p) {
     PASK_MEM_CASE(MEM_GAVG, TimelineScope ts(p.p.tl); gavg_body(p.p))
     PASK_MEM_CASE(MEM_SOFTMAX, TimelineScope ts(p.r.tl); softmax_body(p.r))
     PASK_MEM_CASE(MEM_LAYERNORM, TimelineScope ts(p.r.tl); layernorm_body(p.r))
+    PASK_MEM_CASE(MEM_GEMV, TimelineScope ts(p.v.tl); gemv_body(p.v))
     default: __trap();
   }
 }
@@ -126,6 +127,14 @@ __global__ void __launch_bounds__(256) pask_softmax(const __grid_constant__ RowP
 __global__ void __launch_bounds__(256) pask_layernorm(const __grid_constant__ RowParams p) {
   TimelineScope ts(p.tl);
   layernorm_body(p);
+}
+#endif
+
+#if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_gemv
+// PASK_K_GEMV (D12)
+__global__ void __launch_bounds__(kGemvThreads) pask_gemv(const __grid_constant__ GemvParams p) {
+  TimelineScope ts(p.tl);
+  gemv_body(p);
 }
 #endif
 

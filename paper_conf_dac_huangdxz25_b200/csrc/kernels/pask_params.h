@@ -137,17 +137,38 @@ struct alignas(16) RowParams {
   unsigned long long* tl;  // pask_config.timeline slots (null = off)
 };
 
+// Weight-streaming GEMV (PASK_K_GEMV, D12): y[m][n] = act(sum_k
+// x[m][k] w[n][k] + bias[n] + res[m][n]) for m < M <= 8.  A CTA of 8 warps owns
+// `nc` consecutive columns; warp w takes column w % nc and K slice w / nc of
+// 8 / nc slices; the slices are summed in fixed order (deterministic).
+constexpr int kGemvThreads = 256;
+constexpr unsigned kGemvSmem = 8 * 8 * 8 * 4;  // partials [slice][column][row], dynamic smem
+struct alignas(16) GemvParams {
+  const void* x;      // bf16, row m at x + m * lda (offset applied)
+  const void* w;      // bf16 [N][ldb] (offset applied)
+  const float* bias;  // [N] or null
+  const void* res;    // bf16, same indexing as y, or null
+  void* y;            // bf16, y[m * ldc + n] (offset applied)
+  int64_t lda, ldb, ldc;
+  int32_t M, N, K;
+  int32_t nc_log2;    // columns per CTA: 1 << nc_log2 (1, 2, 4 or 8)
+  int32_t per;        // 16-byte K vectors per slice: ceil(K / 8 / slices)
+  int32_t act;
+  unsigned long long* tl;  // pask_config.timeline slots (null = off)
+};
+
 // Operator-family entry (pask_config.packaging = 2): the memory-bound solutions
 // (layout, depthwise conv, pooling, softmax, LayerNorm) share ONE CUfunction,
 // `pask_mem`, so one code upload makes all of them resident.  The solution's
 // own parameter block sits at offset 0; `kind` selects its body.
-enum MemKind : int32_t { MEM_LAYOUT = 0, MEM_DW, MEM_POOL, MEM_GAVG, MEM_SOFTMAX, MEM_LAYERNORM };
+enum MemKind : int32_t { MEM_LAYOUT = 0, MEM_DW, MEM_POOL, MEM_GAVG, MEM_SOFTMAX, MEM_LAYERNORM, MEM_GEMV };
 struct alignas(16) MemParams {
   union {
     LayoutParams l;
     PoolParams p;
     DwParams d;
     RowParams r;
+    GemvParams v;
   };
   int32_t kind;  // MemKind
 };

@@ -21,6 +21,7 @@ struct Problem {
   int32_t groups = 0, p = 0, q = 0, pool_mode = 0, global = 0;
   int32_t gm = 0, gn = 0, gk = 0, batch = 0;
   int64_t lda = 0, ldb = 0, off_a = 0, off_b = 0;
+  int32_t trans_b = 0, b_weights = 0;  // GEMM: B stored [n][k]; B is the weight operand (w)
   int32_t rows = 0, cols = 0;
 };
 
@@ -68,6 +69,9 @@ constexpr uint32_t kMaxDynSmem = 220u * 1024u;
 // max_cluster: largest split-K cluster the device co-schedules (16 on a full B200)
 GemmTiling gemm_tiling(int32_t M, int32_t N, int32_t K, int32_t batch, int32_t b_major, int32_t c_tma,
                        int32_t persistent_kernel = 0, int32_t max_cluster = 16);
+// s* rule: a GEMM of at most kGemvMaxRows rows with a [N][K] weight operand takes
+// the GEMV solution (PASK_K_GEMV, D12)
+constexpr int32_t kGemvMaxRows = 8;
 // s* rule: a dense conv with more output rows than 148 SMs x 128-row tiles takes
 // the persistent-tile solution (PASK_K_CONV_IGEMM_PT)
 constexpr int64_t kPersistentRows = 148 * 128;

@@ -22,8 +22,8 @@ NCHW, NHWC, ROWMAJOR = 0, 1, 2
 OP_LAYOUT, OP_CONV2D, OP_GEMM, OP_POOL, OP_SOFTMAX, OP_LAYERNORM, OP_ATTENTION = range(7)
 ACT = {"none": 0, "relu": 1, "relu6": 2, "gelu": 3, "tanh": 4}
 K_LAYOUT, K_CONV_IGEMM, K_CONV_1X1, K_CONV_DW, K_POOL, K_POOL_GAVG, K_GEMM, K_SOFTMAX, \
-    K_LAYERNORM, K_ATTENTION, K_CONV_IGEMM_PT = range(11)
-NUM_KERNELS = 11         # generic catalog (PASK_NUM_KERNELS); num_kernels() adds the specialisations
+    K_LAYERNORM, K_ATTENTION, K_CONV_IGEMM_PT, K_GEMV = range(12)
+NUM_KERNELS = 12         # generic catalog (PASK_NUM_KERNELS); num_kernels() adds the specialisations
 HOW = {0: "direct", 1: "reused", 2: "loaded"}
 
 

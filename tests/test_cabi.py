@@ -193,7 +193,7 @@ def test_kernel_function_families():
     """pask_kernel_function: the CUfunction serving each solution per packaging
     (D8).  Packaging 0/1: the solution's own entry; packaging 2: the
     memory-bound family entry or the generic implicit-GEMM entry."""
-    mem = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM}
+    mem = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM, P.K_GEMV}
     contract = {P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
     for k in range(P.num_kernels()):
         assert P.function_name(k, 0) == P.function_name(k, 1) == P.kernel_name(k)

@@ -148,7 +148,29 @@ def linear_spec(m, kin, nout, act="none", res=False, rows=None, seed=4):
     (64, 16384, 32, "none", True, None),    # 16-way split, a full 64-row A box, residual
 ])
 def test_linear_cases(m, kin, nout, act, res, rows):
-    _check_spec(linear_spec(m, kin, nout, act, res, rows))
+    spec = linear_spec(m, kin, nout, act, res, rows)
+    _check_spec(spec)
+    if m <= 8:   # s* there is the GEMV solution (D12): also run the tcgen05 GEMM on it
+        _check_spec(spec, solutions={i: P.K_GEMM for i in range(len(spec["layers"]))})
+
+
+@pytest.mark.parametrize("m,kin,nout,act,res,rows", [
+    (1, 2048, 1000, "none", False, None),   # ResNet-50 FC: 4 columns per CTA, 2 K slices
+    (1, 1280, 1000, "none", False, None),   # MobileNetV2 FC
+    (1, 16384, 10, "none", False, None),    # tiny CNN FC: 10 CTAs of 32 warps, 32 K slices
+    (128, 768, 768, "tanh", False, 1),      # BERT pooler (rows = 1)
+    (8, 512, 33, "gelu", True, None),       # 8 rows, N tail, GELU, residual
+    (3, 64, 300, "relu", True, None),       # K = 64: 8 vectors, most lanes idle
+    (2, 40960, 3, "relu6", False, None),    # K slices of 160 vectors: past the 4 preloaded per lane
+])
+def test_gemv_cases(m, kin, nout, act, res, rows):
+    """PASK_K_GEMV (D12) vs the fp64 linear definition: every layer with
+    <= 8 rows is bound to it (s*), the rest to pask_gemm."""
+    spec = linear_spec(m, kin, nout, act, res, rows)
+    dm, plan = _check_spec(spec)
+    for (i, want, bound, how, lk), L in zip(plan, spec["layers"]):
+        rows_i = L["rows"] if L["rows"] is not None else m
+        assert want == (P.K_GEMV if rows_i <= 8 else P.K_GEMM)
 
 
 def test_attention_batched_gemm():

@@ -127,7 +127,8 @@ def test_family_packaging_bitwise(name):
     o = OP.execution_plan(OP.problems_from_spec(spec))
     assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
     st = ctx.stats()
-    fams = {("mem" if k in (P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM)
+    fams = {("mem" if k in (P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM,
+                            P.K_GEMV)
              else "contract" if k in (P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM) else k) for k in o["loaded"]}
     assert st["kernels_loaded"] == len(fams)
     # both families share one code object; other kernels keep their own
@@ -152,7 +153,7 @@ def test_single_function_packaging_bitwise(name):
     o = OP.execution_plan(OP.problems_from_spec(spec))
     assert [tuple(b) for b in plan] == [tuple(b) for b in o["bindings"]]
     st = ctx.stats()
-    fam = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM,
+    fam = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM, P.K_GEMV,
            P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
     own = set(o["loaded"]) - fam
     assert st["kernels_loaded"] == len(own) + 1

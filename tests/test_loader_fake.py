@@ -42,7 +42,7 @@ MODES = [
 # the fake driver logs it (the memory family entry `pask_mem` is id 63)
 FAM_MEM = 63
 FAM_ALL = 62   # packaging 3 (D10): `pask_all`
-MEM_SOLUTIONS = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM}
+MEM_SOLUTIONS = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM, P.K_GEMV}
 CONTRACT_SOLUTIONS = {P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
 
 
@@ -261,7 +261,8 @@ def test_family_variant_covers_the_plan(name, variant):
     st = ctx.stats()
     ctx.close()
     mask = B.FAMILY_VARIANTS[f"pask_families_{variant}"]
-    kinds = {P.K_LAYOUT: 0, P.K_CONV_DW: 1, P.K_POOL: 2, P.K_POOL_GAVG: 3, P.K_SOFTMAX: 4, P.K_LAYERNORM: 5}
+    kinds = {P.K_LAYOUT: 0, P.K_CONV_DW: 1, P.K_POOL: 2, P.K_POOL_GAVG: 3, P.K_SOFTMAX: 4, P.K_LAYERNORM: 5,
+             P.K_GEMV: 6}
     need = {kinds[k] for b in plan for k in (b[1], b[2]) if k in kinds}
     assert all((mask >> kd) & 1 for kd in need)
     smaller = [m for v, m in B.FAMILY_VARIANTS.items() if bin(m).count("1") < bin(mask).count("1")]
@@ -321,10 +322,12 @@ def test_overlapping_tensors_run_on_one_stream():
 
 
 def test_cluster_size_capped_by_device_occupancy():
-    """the tiny CNN's FC (M = 1, K = 16384) plans a 16-CTA split-K
-    cluster; where the device cannot co-schedule one the node is lowered again
+    """the tiny CNN's FC (M = 1, K = 16384) on the tcgen05 GEMM plans a
+    16-CTA split-K cluster; where the device cannot co-schedule one the node is lowered again
     with at most 8, before it is launched."""
     spec, _ = build_model("tiny_cnn")
+    fc = [i for i, L in enumerate(spec["layers"]) if L["op"] == "linear"][0]
+    sol = {fc: P.K_GEMM}       # the FC's s* is the GEMV solution; force the tcgen05 GEMM
     for occ, want in ((1, 16), (0, 8)):
         P.test_fake_driver(True)
         P.test_fake_knob(P.FAKE_OCCUPANCY, occ)
@@ -332,7 +335,7 @@ def test_cluster_size_capped_by_device_occupancy():
             P.test_fake_driver(True)
             P.test_fake_knob(P.FAKE_OCCUPANCY, occ)
             ctx = P.Context(0, P.config(**mode))
-            ctx.load_model(DeviceModel(spec, alloc=False).graph)
+            ctx.load_model(DeviceModel(spec, alloc=False, solutions=sol).graph)
             ctx.infer(0)
             ctx.sync()
             st = ctx.stats()

@@ -41,17 +41,22 @@ def test_mbv2_prefix_hand_trace(golden):
 
 
 def test_full_model_counts_match_survey():
-    """SURVEY.md §8(a) a3 (computed independently by the survey from the candidate catalog)."""
+    """SURVEY.md §8(a) a3 (computed independently by the survey from the candidate
+    catalog), with DESIGN.md D12's GEMV solution added to the catalog: the FC
+    layers of C1-C3 (M = 1) have s* = pask_gemv instead of pask_gemm -- the GEMM
+    category is still empty at their query, so the query / hit / lookup counts
+    are the survey's -- and BERT's pooler (M = 1) now queries the GEMM category
+    and reuses the loaded pask_gemm (one more query, one hit, one lookup)."""
     expect = {
-        "tiny_cnn": (["pask_layout", "pask_conv_igemm", "pask_pool", "pask_gemm",
+        "tiny_cnn": (["pask_layout", "pask_conv_igemm", "pask_pool", "pask_gemv",
                       "pask_softmax"], 5, 0, 0),
-        "resnet50": (["pask_layout", "pask_conv_igemm", "pask_pool", "pask_gemm",
+        "resnet50": (["pask_layout", "pask_conv_igemm", "pask_pool", "pask_gemv",
                       "pask_softmax"], 39, 34, 34),
         "mobilenet_v2": (["pask_layout", "pask_conv_igemm", "pask_conv_dw", "pask_pool_gavg",
-                          "pask_gemm", "pask_softmax"], 40, 34, 34),
-        "bert_base": (["pask_layernorm", "pask_gemm", "pask_softmax"], 3, 0, 0),
+                          "pask_gemv", "pask_softmax"], 40, 34, 34),
+        "bert_base": (["pask_layernorm", "pask_gemm", "pask_softmax"], 4, 1, 1),
         # NEXT #4: qk -> softmax -> pv fused; the attention solution replaces softmax
-        "bert_base_fa": (["pask_layernorm", "pask_gemm", "pask_attention"], 3, 0, 0),
+        "bert_base_fa": (["pask_layernorm", "pask_gemm", "pask_attention"], 4, 1, 1),
     }
     for name, (loaded, q, h, lk) in expect.items():
         spec, _ = build_model(name)
@@ -68,7 +73,7 @@ def test_full_model_counts_match_survey():
     spec, _ = build_model("resnet50", batch=128)
     pl = P.execution_plan(P.problems_from_spec(spec))
     assert [P.KERNEL_NAMES[k] for k in pl["loaded"]] == [
-        "pask_layout", "pask_conv_igemm_pt", "pask_pool", "pask_gemm", "pask_softmax"]
+        "pask_layout", "pask_conv_igemm_pt", "pask_pool", "pask_gemm", "pask_softmax"]   # FC M = 128: gemm
     # no reuse: ResNet-50 loads 7 distinct s* (adds conv_1x1 and gavg), MobileNetV2 7
     for name, n in (("resnet50", 7), ("mobilenet_v2", 7)):
         spec, _ = build_model(name)
@@ -115,7 +120,8 @@ def _random_problem(rng):
         return p
     p = dict(P._ZERO)
     k = rng.choice([64, 60])
-    p.update(op=P.GEMM, gm=4, gn=8, gk=k, batch=1, lda=k, ldb=k)
+    p.update(op=P.GEMM, gm=rng.choice([4, 16]), gn=8, gk=k, batch=1, lda=k, ldb=k, trans_b=1,
+             b_weights=rng.choice([0, 1]))
     return p
 
 
@@ -208,3 +214,23 @@ def test_tuned_catalog_covers_every_config_conv_and_plans():
     assert len(pask["loaded"]) == 21 and pask["hits"] == 1      # only gavg -> pool
     for (i, want, bound, how, lk) in pask["bindings"]:
         assert P.is_applicable(bound, probs[i])
+
+
+def test_gemv_predicate_and_choice():
+    """DESIGN.md D12: the GEMV solution is s* (and applicable) exactly for a
+    single GEMM with a weight operand stored [N][K] and 1..8 rows, K, lda, ldb and
+    the offsets multiples of 8 (16-byte vectors); otherwise s* stays pask_gemm,
+    which is applicable to every such GEMM too (so the pooler can reuse it)."""
+    base = dict(P._ZERO)
+    base.update(op=P.GEMM, gm=1, gn=1000, gk=2048, batch=1, lda=2048, ldb=2048, trans_b=1, b_weights=1)
+    assert P.static_choice(base) == P.K_GEMV
+    assert P.is_applicable(P.K_GEMM, base)
+    for m in (1, 2, 8):
+        assert P.static_choice({**base, "gm": m}) == P.K_GEMV
+    for bad in (dict(gm=9), dict(gm=0), dict(batch=2), dict(trans_b=0), dict(b_weights=0), dict(gk=2044),
+                dict(lda=2050), dict(ldb=2052), dict(off_a=4), dict(off_b=12), dict(gn=0)):
+        q = {**base, **bad}
+        assert not P.is_applicable(P.K_GEMV, q), bad
+        if q["gm"] >= 1 and q["gn"] >= 1 and q["gk"] % 8 == 0:
+            assert P.static_choice(q) == P.K_GEMM, bad
+    assert P.CATEGORY[P.K_GEMV] == P.CATEGORY[P.K_GEMM]
