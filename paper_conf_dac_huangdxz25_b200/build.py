@@ -63,13 +63,18 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # LayerNorm 5, GEMV 6); the runtime loads the smallest covering the model's solutions
 # (dwg = depthwise + global pool without the windowed pool: MobileNetV2).
 # Packaging 3 (D10): both families behind the single entry `pask_all`.
+# Each variant also compiles only some contraction paths (PASK_GEMM_FEAT, bit per
+# GemmFeat of conv_gemm.cuh: split-K 1, MN-major B 2, staged epilogue 4, scalar
+# epilogue 8, GELU / tanh 16, cp.async gather 32, TMA im2col 64; D13).
 # Smallest first: the runtime takes the first variant covering the plan (the
 # table is generated into _build/spec_catalog.h as PASK_FAMILY_VARIANTS).
-FAMILY_VARIANTS = {"pask_families_tf": 0x70, "pask_families_dwg": 0x5b, "pask_families_cnn": 0x5d,
-                   "pask_families_dw": 0x5f, "pask_families": 0x7f}
+FAMILY_VARIANTS = {"pask_families_tf": (0x70, 0x17), "pask_families_dwg": (0x5b, 0x25),
+                   "pask_families_cnn": (0x5d, 0x61), "pask_families_dw": (0x5f, 0x7f),
+                   "pask_families": (0x7f, 0x7f)}
 EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"],
                  "pask_primer": ["pask_primer"]}   # pask_create's driver primer (not a solution)
-EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}"] for k, m in FAMILY_VARIANTS.items()}
+EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}", f"-DPASK_GEMM_FEAT={g:#x}"]
+                 for k, (m, g) in FAMILY_VARIANTS.items()}
 
 # The "tuned library": one specialised conv solution per distinct
 # dense-conv problem (R, S, stride, pad, dilation, input channels C) of configs
@@ -108,9 +113,10 @@ def _gen_spec_sources():
     host += ["    {%d, %d, %d, %d, %d, %d, \"%s\"}," % (*sp, spec_name(sp)) for sp in SPECS]
     host += ["};", "}  // namespace pask", ""]
     host += ["#define PASK_SPEC_IMAGES(X) \\"] + [f"  X({spec_name(sp)}) \\" for sp in SPECS] + [""]
-    host += ["// packaging 2 families variants (name, memory-case mask), smallest first",
+    host += ["// packaging 2 families variants (name, memory-case mask, contraction-path mask),",
+             "// smallest first",
              "#define PASK_FAMILY_VARIANTS(X) \\"] + \
-        [f"  X({k}, {m:#x}) \\" for k, m in FAMILY_VARIANTS.items()] + ["", ""]
+        [f"  X({k}, {m:#x}, {g:#x}) \\" for k, (m, g) in FAMILY_VARIANTS.items()] + ["", ""]
     for path, text in ((os.path.join(BUILD, "spec_kernels.inc"), "".join(ker)),
                        (os.path.join(BUILD, "spec_catalog.h"), "\n".join(host))):
         old = open(path).read() if os.path.exists(path) else None

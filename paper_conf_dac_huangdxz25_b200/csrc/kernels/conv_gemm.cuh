@@ -39,6 +39,28 @@
 
 namespace pask {
 
+// Paths compiled into the one-tile contraction body (conv_gemm_body).  The
+// operator-families objects come in variants (build.py FAMILY_VARIANTS) that
+// compile only the paths their models' plans use, so a model uploads less code
+// (an upload costs ~1.1 us per KB of SASS, D8 / D13); the host picks
+// the smallest variant covering every contraction node, and a launch that asks
+// for a path compiled out traps instead of computing something else.
+enum GemmFeat : unsigned {
+  GF_SPLITK = 1,    // split-K thread-block clusters (DSMEM reduction)
+  GF_MN_B = 2,      // MN-major B operand (attention PV)
+  GF_STAGED = 4,    // staged epilogue + TMA tensor store (c_tma = 1)
+  GF_SCALAR = 8,    // scalar epilogue for unaligned rows (c_tma = 0)
+  GF_SLOWACT = 16,  // GELU / tanh epilogue
+  GF_GATHER = 32,   // A_GATHER implicit im2col by cp.async
+  GF_IM2COL = 64,   // A_IM2COL implicit im2col by TMA
+  GF_ALL = 127
+};
+#ifndef PASK_GEMM_FEAT
+#define PASK_GEMM_FEAT 127
+#endif
+constexpr unsigned kGemmFeat = PASK_GEMM_FEAT;
+__device__ __forceinline__ constexpr bool gfeat(unsigned f) { return (kGemmFeat & f) != 0; }
+
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
@@ -53,7 +75,7 @@ __device__ __forceinline__ void act16(float (&v)[16], int act) {
   } else if (act == 2) {
 #pragma unroll
     for (int i = 0; i < 16; ++i) v[i] = fminf(fmaxf(v[i], 0.f), 6.f);
-  } else if (act >= 3) {
+  } else if (act >= 3 && gfeat(GF_SLOWACT)) {
 #pragma unroll
     for (int i = 0; i < 16; ++i) v[i] = act_slow(v[i], act);
   }
@@ -115,10 +137,10 @@ __device__ __forceinline__ void epi16(const EpiArgs& p, uint32_t sbias, uint32_t
     v[4 * q4 + 2] += bb.z;
     v[4 * q4 + 3] += bb.w;
   }
-  if (p.c_tma) {
+  if (p.c_tma || !gfeat(GF_SCALAR)) {
     const uint32_t a0 = ro_addr(ro, lb, row, cb);
     const uint32_t a1 = ro_addr(ro, lb, row, cb + 8);
-    if (p.res) {
+    if (p.res) {  // the residual tile was TMA-loaded into the staging smem
       float f0[8], f1[8];
       unpack_bf16x8(lds_u4(a0), f0);
       unpack_bf16x8(lds_u4(a1), f1);
@@ -133,7 +155,7 @@ __device__ __forceinline__ void epi16(const EpiArgs& p, uint32_t sbias, uint32_t
                                 pack_bf16x2(v[6], v[7]));
     const uint4 w1 = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
                                 pack_bf16x2(v[14], v[15]));
-    if (p.c_tma == 2) {
+    if (p.c_tma == 2 || !gfeat(GF_STAGED)) {
       // direct epilogue: the 32 B of one output row in a single 256-bit store from
       // registers (N % 16 == 0, 32-byte aligned rows; one-tile kernel only)
       if (n0 + cb < p.N)
@@ -208,7 +230,15 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int t = threadIdx.x;
   const int stages = p.stages;
   const int bn = p.bn;
-  const int splits = p.splits;
+  // a path compiled out of this families variant (GemmFeat) must never be asked for
+  if (kGemmFeat != GF_ALL &&
+      ((!gfeat(GF_SPLITK) && p.splits > 1) || (!gfeat(GF_MN_B) && p.b_major != 0) ||
+       (!gfeat(GF_STAGED) && p.c_tma == 1) || (!gfeat(GF_SCALAR) && p.c_tma == 0) ||
+       (!gfeat(GF_SLOWACT) && p.act >= 3) || (!gfeat(GF_GATHER) && kAllowGather && p.a_mode == A_GATHER) ||
+       (!gfeat(GF_IM2COL) && kAllowGather && p.a_mode == A_IM2COL)))
+    __trap();
+  const int splits = gfeat(GF_SPLITK) ? p.splits : 1;
+  const int b_major = gfeat(GF_MN_B) ? p.b_major : 0;
   constexpr uint32_t kABytes = kBM * kBK * 2;  // 16 KB
   const uint32_t b_bytes = static_cast<uint32_t>(bn) * kBK * 2;
   const uint32_t stage_bytes = kABytes + b_bytes;
@@ -232,8 +262,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const uint32_t recv = smem_base + ring_bytes;  // slot s: rows [s*rows_per, (s+1)*rows_per)
 
   const int a_mode = Geo::amode(p);
-  const bool gather = kAllowGather && (a_mode == A_GATHER);
-  const bool im2col = kAllowGather && (a_mode == A_IM2COL);
+  const bool gather = kAllowGather && gfeat(GF_GATHER) && (a_mode == A_GATHER);
+  const bool im2col = kAllowGather && gfeat(GF_IM2COL) && (a_mode == A_IM2COL);
   const int gR = Geo::R(p), gS = Geo::S(p), gSH = Geo::SH(p), gSW = Geo::SW(p);
   const int gPH = Geo::PH(p), gPW = Geo::PW(p), gDH = Geo::DH(p), gDW = Geo::DW(p), gC = Geo::C(p);
   (void)gR;
@@ -326,7 +356,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const uint32_t sb = smem_base + i * stage_bytes + kABytes;
         const int kb = kb_begin + i;
         mbar_arrive_expect_tx(full0 + 8 * i, b_bytes + (gather ? 0u : a_tx));
-        if (p.b_major == 0) {
+        if (b_major == 0) {
           tma_load_3d(sb, &p.tmap_b, full0 + 8 * i, kb * kBK, n0, b);
         } else {
 #pragma unroll 1
@@ -366,7 +396,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, b);
         }
         if (!b_done) {
-          if (p.b_major == 0) {
+          if (b_major == 0) {
             tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, b);
           } else {
 #pragma unroll 1
@@ -396,7 +426,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         for (int k = 0; k < kBK / 16; ++k) {
           // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row
           const uint64_t adesc = umma_desc_sw128(sa + k * 32, 16, 1024);
-          const uint64_t bdesc = (p.b_major == 0)
+          const uint64_t bdesc = (b_major == 0)
                                      ? umma_desc_sw128(sb + k * 32, 16, 1024)
                                      // MN-major: +16 K rows of 128 B; 64-wide N chunks 8 KB apart
                                      : umma_desc_sw128(sb + k * 2048, 8192, 1024);
@@ -610,7 +640,7 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
       if (more) tmem_ld_wait(r);
     }
     if (trace && t == 0) trace[6] = stamp();
-    if (p.c_tma == 1) {
+    if (gfeat(GF_STAGED) && p.c_tma == 1) {
       fence_proxy_async_smem();  // staged bf16 tile -> TMA store (async proxy)
       named_bar_sync(1, kEpiThreads);
       if (t == 0 && slice_rows > 0) {

@@ -108,7 +108,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1) pask_gemm(const __grid_consta
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_attention
 // PASK_K_ATTENTION: fused QK^T -> softmax -> PV (tcgen05, scores in TMEM)
-__global__ void __launch_bounds__(192, 1) pask_attention(const __grid_constant__ AttnParams p) {
+__global__ void __launch_bounds__(320, 1) pask_attention(const __grid_constant__ AttnParams p) {
   TimelineScope ts(p.tl);
   attention_body(p);
 }
