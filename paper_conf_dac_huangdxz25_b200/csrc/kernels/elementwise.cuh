@@ -22,9 +22,15 @@ __device__ __forceinline__ float warp_max(float v) {
 // Activation over 8 values: ReLU / ReLU6 inline, GELU / tanh out of line (rare
 // on the memory-bound path; keeps the code object small -- uploads cost ~1.1 us
 // per KB of SASS).  Same arithmetic as apply_act either way.
-__device__ __noinline__ void act8_slow(float (&v)[8], int act) {
+struct F8 {
+  float v[8];
+};
+// by value in registers (a reference parameter would put the array on the stack
+// and give every memory kernel a local-memory frame)
+__device__ __noinline__ F8 act8_slow(F8 x, int act) {
 #pragma unroll
-  for (int i = 0; i < 8; ++i) v[i] = apply_act(v[i], act);
+  for (int i = 0; i < 8; ++i) x.v[i] = apply_act(x.v[i], act);
+  return x;
 }
 __device__ __forceinline__ void act8(float (&v)[8], int act) {
   if (act == 1) {
@@ -34,7 +40,12 @@ __device__ __forceinline__ void act8(float (&v)[8], int act) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) v[i] = fminf(fmaxf(v[i], 0.f), 6.f);
   } else if (act >= 3) {
-    act8_slow(v, act);
+    F8 x;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x.v[i] = v[i];
+    x = act8_slow(x, act);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = x.v[i];
   }
 }
 

@@ -22,9 +22,12 @@ __device__ __forceinline__ unsigned long long globaltimer() {
 // %globaltimer ns (start slot tl[0], end slot tl[kTimelineStride]).  Thread 0 of
 // each CTA stamps on entry and when it leaves the body; two relaxed 64-bit
 // atomics per CTA, none when tl is null (the default).
+// The scope holds a reference to the __grid_constant__ parameter field, not
+// its value, so the pointer is re-read from the parameter bank at the end
+// instead of occupying two registers across the kernel body.
 struct TimelineScope {
-  unsigned long long* tl;
-  __device__ __forceinline__ explicit TimelineScope(unsigned long long* p) : tl(p) {
+  unsigned long long* const& tl;
+  __device__ __forceinline__ explicit TimelineScope(unsigned long long* const& p) : tl(p) {
     if (tl != nullptr && threadIdx.x == 0) atomicMin(tl, globaltimer());
   }
   __device__ __forceinline__ ~TimelineScope() {
