@@ -137,19 +137,27 @@ def breakdown(samples: list[dict]) -> dict:
       load       plan done -> every planned kernel uploaded (encode overlaps it)
       issue      uploads done -> first launch issued (infer entry, first launch)
       gpu_busy   union of the kernels' [start, end] intervals (timeline stamps)
-      gpu_idle   first launch -> last kernel end, minus busy (issue-paced gaps)
+      gpu_idle   first launch -> end of the event span, minus busy (issue-paced
+                 gaps; for schemes that load during the issue, the GPU waiting
+                 for those loads)
       other      the rest of the window (sync return)
+    The six parts sum to the cold wall.
     and GPU utilisation = gpu_busy / cold wall (Fig. 6(b))."""
     rows = []
     for s in samples:
         cold = s["cold_us"]
         plan = s["plan_us"]
-        load = max(0.0, s["t_load_done_us"] - plan)
-        issue = max(0.0, s["t_first_launch_us"] - s["t_load_done_us"])
-        span = s["gpu_span_us"]
-        busy = min(s["gpu_busy_us"], span)
-        other = cold - plan - load - issue - span
-        rows.append({"plan": plan, "load": load, "issue": issue, "gpu_busy": busy, "gpu_idle": span - busy,
+        first = s["t_first_launch_us"]
+        # schemes that load during the issue (reactive, loader thread, interleave):
+        # loads after the first launch show up as GPU idle (the GPU waits for them)
+        ld = min(s["t_load_done_us"], first)
+        load = max(0.0, ld - plan)
+        issue = max(0.0, first - max(plan, ld))
+        window = cold - first                              # first launch -> t1
+        busy = min(s["gpu_busy_us"], window)
+        other = max(0.0, window - s["gpu_span_us"])        # outside the event span: the sync return
+        idle = max(0.0, window - busy - other)
+        rows.append({"plan": plan, "load": load, "issue": issue, "gpu_busy": busy, "gpu_idle": idle,
                      "other": other, "cold": cold, "util": busy / cold if cold else 0.0})
     return {k: round(statistics.median(r[k] for r in rows), 1 if k != "util" else 4) for k in rows[0]}
 
