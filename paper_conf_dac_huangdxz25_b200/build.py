@@ -68,12 +68,18 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # epilogue 8, GELU / tanh 16, cp.async gather 32, TMA im2col 64; D13).
 # Smallest first: the runtime takes the first variant covering the plan (the
 # table is generated into _build/spec_catalog.h as PASK_FAMILY_VARIANTS).
-FAMILY_VARIANTS = {"pask_families_tf": (0x70, 0x17), "pask_families_dwg": (0x5b, 0x25),
-                   "pask_families_cnn": (0x5d, 0x61), "pask_families_dw": (0x5f, 0x7f),
+# The CNN variants also drop softmax's register-resident row path (their one
+# softmax row of 10 / 1000 classes takes the two-pass loop: same arithmetic,
+# bitwise equal) -- PASK_SOFTMAX_REG.
+FAMILY_VARIANTS = {"pask_families_tf": (0x30, 0x17), "pask_families_dwg": (0x5b, 0x25),
+                   "pask_families_cnn": (0x55, 0x61), "pask_families_dw": (0x5f, 0x7f),
                    "pask_families": (0x7f, 0x7f)}
+FAMILY_SOFTMAX_REG = {"pask_families_tf": 1, "pask_families_dwg": 0, "pask_families_cnn": 0,
+                      "pask_families_dw": 1, "pask_families": 1}
 EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"],
                  "pask_primer": ["pask_primer"]}   # pask_create's driver primer (not a solution)
-EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}", f"-DPASK_GEMM_FEAT={g:#x}"]
+EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}", f"-DPASK_GEMM_FEAT={g:#x}",
+                     f"-DPASK_SOFTMAX_REG={FAMILY_SOFTMAX_REG[k]}"]
                  for k, (m, g) in FAMILY_VARIANTS.items()}
 
 # The "tuned library": one specialised conv solution per distinct

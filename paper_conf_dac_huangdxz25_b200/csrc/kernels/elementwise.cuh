@@ -292,6 +292,11 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
 // One warp per row.  Pass 1: online max / sum of exp(scale*x - max) in fp32;
 // pass 2: write exp(scale*x - max) / sum as bf16.
 constexpr int kSmRegChunks = 4;  // 16 B chunks per lane kept in registers (rows <= 1024)
+// the register-resident path for short rows (BERT's 1536 attention rows per
+// layer); families variants for models with one softmax row compile it out
+#ifndef PASK_SOFTMAX_REG
+#define PASK_SOFTMAX_REG 1
+#endif
 __device__ __forceinline__ void softmax_body(const RowParams& p) {
   pdl_wait();
   pdl_launch_dependents();
@@ -302,7 +307,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
   const bool vec = (p.cols & 7) == 0;
   float m = -INFINITY, s = 0.f;
-  if (vec && p.cols <= 256 * kSmRegChunks) {
+  if (PASK_SOFTMAX_REG && vec && p.cols <= 256 * kSmRegChunks) {
     // short rows (BERT attention: 128, classifiers: 1000): the row stays in
     // registers, one load round trip; same arithmetic order as the loop below
     float f[kSmRegChunks][8];

@@ -245,10 +245,9 @@ def test_branches_issue_side_nodes_after_their_producer(name):
                                           ("bert_base", "tf"), ("bert_base_fa", "tf")])
 def test_family_variant_covers_the_plan(name, variant):
     """Packaging 2 (D8): the families object is loaded in the smallest
-    variant whose memory-bound cases cover every solution the plan desires or
-    binds (CNN: layout / pool / global-average pool / softmax; layout /
-    depthwise / global-average pool / softmax for MobileNetV2; softmax /
-    LayerNorm for BERT) and whose contraction entry compiles the paths the
+    variant whose memory-bound cases cover every solution the plan binds (CNN:
+    layout / pool / softmax / GEMV; layout / depthwise / global-average pool /
+    softmax / GEMV for MobileNetV2; softmax / LayerNorm for BERT) and whose contraction entry compiles the paths the
     plan's contraction nodes take (D13: split-K / gather / im2col for
     the CNNs, staged epilogues for MobileNetV2's N = 24 layers, MN-major B and
     GELU for BERT); one code object, whose bytes are that variant's image
@@ -266,7 +265,7 @@ def test_family_variant_covers_the_plan(name, variant):
     mask = B.FAMILY_VARIANTS[f"pask_families_{variant}"][0]
     kinds = {P.K_LAYOUT: 0, P.K_CONV_DW: 1, P.K_POOL: 2, P.K_POOL_GAVG: 3, P.K_SOFTMAX: 4, P.K_LAYERNORM: 5,
              P.K_GEMV: 6}
-    need = {kinds[k] for b in plan for k in (b[1], b[2]) if k in kinds}
+    need = {kinds[b[2]] for b in plan if b[2] in kinds}     # the bound solutions (D13)
     assert all((mask >> kd) & 1 for kd in need)
     # variants are tried smallest first; the ones before the chosen one lack a
     # memory case or a contraction path (D13) the plan needs
