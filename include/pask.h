@@ -206,8 +206,8 @@ typedef struct {
                              resident; the plan (Algorithm 1) is unchanged, kernels_loaded
                              counts the uploaded functions; the families object is loaded
                              in the smallest variant whose memory cases cover every
-                             solution the plan desires or binds (all / CNN / CNN +
-                             depthwise / transformer);
+                             solution the plan binds and whose contraction entry compiles
+                             every path the plan's contraction nodes take (D13);
                          3 = one CUfunction `pask_all` for both families (D10:
                              one upload, measured slower on the hot path; not the default) */
   int32_t interleave; /* 0 = load-first (default): the first inference launches once every
