@@ -34,6 +34,7 @@ struct Tuning {
   bool join_no_pdl = false;        // branches: drop PDL after a join wait
   bool direct_one_stream = false;  // branches: direct issue on one stream
   bool no_event_warm = false;      // pask_create: do not pre-record the timing events
+  bool parallel_upload = false;    // packaging 2: helper uploads the contraction family concurrently
   // device phase trace (experiment builds only)
   int trace_node = -2;             // node index, -1 = all, -2 = off
   uint64_t trace_ptr = 0;          // device address of the trace buffer
