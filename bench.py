@@ -177,7 +177,8 @@ def replica_summary(per_rank_conc, solo, per_rank_hot_ms, batch):
     for r, trials in enumerate(per_rank_conc):
         c = [t["cold_us"] / 1e3 for t in trials]
         per.append({"rank": r, "cold_med_ms": round(statistics.median(c), 3), "cold_max_ms": round(max(c), 3),
-                    "trials": len(c), "kernels_loaded": sorted({int(t["kernels_loaded"]) for t in trials})})
+                    "trials": len(c), "kernels_loaded": sorted({int(t["kernels_loaded"]) for t in trials}),
+                    "cold_ms": [round(v, 3) for v in c]})
     all_conc = [t["cold_us"] / 1e3 for trials in per_rank_conc for t in trials]
     solo_ms = [t["cold_us"] / 1e3 for t in solo]
     cn = statistics.median(all_conc)
@@ -385,6 +386,9 @@ def main():
     from scripts import cold_samples as cs
 
     pbuild.build()
+    # one replica per GPU (LOCAL_RANK -> device); on a box with fewer GPUs than
+    # ranks (a harness check on one GPU) ranks share devices round-robin
+    local_rank = local_rank % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     stream = torch.cuda.current_stream(dev)
