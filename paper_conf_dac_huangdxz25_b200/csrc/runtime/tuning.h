@@ -23,6 +23,7 @@ struct Tuning {
   int bn32_tiles = 8;     // unsplittable layers with <= this many tiles take 32-wide N tiles
   int fine_ctas = 32;     // grids below this many CTAs with K <= fine_max_k retile finer (0: off)
   int fine_max_k = 1024;
+  int fine_max_mtiles = 8;
   // lowering (pask.cpp)
   int gather_lag = 2;     // A_GATHER: k-blocks of cp.async in flight before publishing a slot
   int pre_b = 0;          // weight k-blocks fetched before griddepcontrol.wait (0 = whole ring)
