@@ -10,6 +10,12 @@
 
 using namespace pask;
 
+// resident CTAs per SM the one-tile contraction entries are compiled for
+// (register budget); experiment builds may ask for 2
+#ifndef PASK_GEMM_MIN_BLOCKS
+#define PASK_GEMM_MIN_BLOCKS 1
+#endif
+
 static_assert(kTimelineStride == 4096, "TimelineScope (ptx.cuh) hard-codes the end-slot offset");
 
 // PASK_MEM_MASK (bit per MemKind) selects the memory-family cases compiled into
@@ -51,7 +57,7 @@ __global__ void __launch_bounds__(256) pask_layout(const __grid_constant__ Layou
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_conv_igemm
 // PASK_K_CONV_IGEMM: generic implicit-GEMM conv (A by gather, or TMA for 1x1 s1 p0)
-__global__ void __launch_bounds__(kGemmThreads, 1) pask_conv_igemm(const __grid_constant__ GemmParams p) {
+__global__ void __launch_bounds__(kGemmThreads, PASK_GEMM_MIN_BLOCKS) pask_conv_igemm(const __grid_constant__ GemmParams p) {
   TimelineScope ts(p.tl);
   conv_gemm_body<true>(p);
 }
@@ -68,7 +74,7 @@ __global__ void __launch_bounds__(kGemmThreadsPT, 1) pask_conv_igemm_pt(const __
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_conv_1x1
 // PASK_K_CONV_1X1: specialised 1x1 / stride 1 / pad 0 conv (A by TMA only)
-__global__ void __launch_bounds__(kGemmThreads, 1) pask_conv_1x1(const __grid_constant__ GemmParams p) {
+__global__ void __launch_bounds__(kGemmThreads, PASK_GEMM_MIN_BLOCKS) pask_conv_1x1(const __grid_constant__ GemmParams p) {
   TimelineScope ts(p.tl);
   conv_gemm_body<false>(p);
 }
@@ -100,7 +106,7 @@ __global__ void __launch_bounds__(128) pask_pool_gavg(const __grid_constant__ Po
 
 #if !defined(PASK_ONLY_KERNEL) || PASK_ONLY_KERNEL_pask_gemm
 // PASK_K_GEMM: batched GEMM (A K-major by TMA; B K- or MN-major by TMA)
-__global__ void __launch_bounds__(kGemmThreads, 1) pask_gemm(const __grid_constant__ GemmParams p) {
+__global__ void __launch_bounds__(kGemmThreads, PASK_GEMM_MIN_BLOCKS) pask_gemm(const __grid_constant__ GemmParams p) {
   TimelineScope ts(p.tl);
   conv_gemm_body<false>(p);
 }

@@ -24,6 +24,7 @@ struct Tuning {
   int fine_ctas = 32;     // grids below this many CTAs with K <= fine_max_k retile finer (0: off)
   int fine_max_k = 1024;
   int fine_max_mtiles = 8;
+  int smem_budget_kb = 220;  // dynamic smem a contraction CTA may use (ring = what is left)
   // lowering (pask.cpp)
   int gather_lag = 2;     // A_GATHER: k-blocks of cp.async in flight before publishing a slot
   int pre_b = 0;          // weight k-blocks fetched before griddepcontrol.wait (0 = whole ring)
