@@ -332,7 +332,11 @@ int main(int argc, char** argv) {
   }
   for (size_t i = 0; i < im.inputs.size(); ++i) {  // the graph inputs' data
     const int32_t b = im.input_blob[i];
+    if (b >= static_cast<int32_t>(im.blob_bytes.size()) || im.inputs[i] < 0 ||
+        im.inputs[i] >= static_cast<int32_t>(im.tensors.size()))
+      die("bad input reference in model image");
     const pask_tensor& t = im.tensors[im.inputs[i]];
+    if (b >= 0 && im.blob_bytes[b] < tensor_bytes(t)) die("input blob smaller than its tensor");
     if (b >= 0) ck(cu.h2d(base + t_off[im.inputs[i]], im.data.data() + im.blob_off[b], tensor_bytes(t)), "upload input");
   }
   CUdeviceptr flush = 0;
