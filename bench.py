@@ -386,6 +386,33 @@ def main():
     from scripts import cold_samples as cs
 
     pbuild.build()
+
+    # ---------------- cold in fresh native processes (N = 1; with replicas the
+    # concurrent trials below are the measurement), taken BEFORE this process
+    # creates its CUDA context, so every sample is the only context on the GPU
+    main_cold, configs_detail = None, {}
+    if world == 1 and args.cold_samples > 0:
+        cfg = bench_cfg(args)
+        image = cs.write_image(args.model, batch=args.batch)
+        try:
+            main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
+            main_cold["cold_no_prefault"] = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1},
+                                                                   args.cold_samples))
+            main_cold["cold_no_prime"] = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1}, args.cold_samples))
+            py = [cs.run_py_child(args.model, cfg, args.batch) for _ in range(args.py_cold_samples)]
+            main_cold["cold_python_process"] = cs.summarize(py) if py else None
+        finally:
+            os.unlink(image)
+        if not args.no_configs and args.batch == 1:
+            for m in CONFIG_MODELS:
+                if m == args.model:
+                    continue
+                image = cs.write_image(m)
+                try:
+                    configs_detail[m] = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, True)
+                finally:
+                    os.unlink(image)
+
     # one replica per GPU (LOCAL_RANK -> device); on a box with fewer GPUs than
     # ranks (a harness check on one GPU) ranks share devices round-robin
     local_rank = local_rank % max(1, torch.cuda.device_count())
@@ -623,45 +650,24 @@ def main():
             dist.destroy_process_group()
         return
 
-    # ---------------- cold in fresh native processes (N = 1; with replicas the
-    # concurrent trials above are the measurement)
-    headline, configs_detail, main_cold = {}, {}, None
-    if world == 1 and args.cold_samples > 0:
-        cfg = bench_cfg(args)
-        image = cs.write_image(args.model, batch=args.batch)
-        try:
-            main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
-            nopf = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1}, args.cold_samples))
-            main_cold["cold_no_prefault"] = nopf
-            nopr = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1}, args.cold_samples))
-            main_cold["cold_no_prime"] = nopr
-            py = [cs.run_py_child(args.model, cfg, args.batch) for _ in range(args.py_cold_samples)]
-            main_cold["cold_python_process"] = cs.summarize(py) if py else None
-        finally:
-            os.unlink(image)
-        c = main_cold["cold"]
+    # ---------------- headline: the fresh-process cold samples taken above, with
+    # this process's hot numbers for the main config
+    headline = {}
+    if main_cold is not None:
+        c, nopf, nopr = main_cold["cold"], main_cold["cold_no_prefault"], main_cold["cold_no_prime"]
+        pyc = main_cold["cold_python_process"]
         headline[args.model] = headline_entry(
             c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"], hot_max, direct_max, main_cold["breakdown"],
             c["kernels_loaded"], main_cold["launches"],
             {"nopf_ms": [round(nopf["median_us"] / 1e3, 3), round(nopf["p90_us"] / 1e3, 3)],
              "noprime_ms": [round(nopr["median_us"] / 1e3, 3), round(nopr["p90_us"] / 1e3, 3)],
-             "py_ms": ([round(main_cold["cold_python_process"]["median_us"] / 1e3, 3),
-                        round(main_cold["cold_python_process"]["p90_us"] / 1e3, 3),
-                        main_cold["cold_python_process"]["n"]] if py else None)})
-        if not args.no_configs and args.batch == 1:
-            for m in CONFIG_MODELS:
-                if m == args.model:
-                    continue
-                image = cs.write_image(m)
-                try:
-                    blk = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, True)
-                finally:
-                    os.unlink(image)
-                configs_detail[m] = blk
-                c = blk["cold"]
-                headline[m] = headline_entry(c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"],
-                                             blk["hot_graph_us"] / 1e3, blk["hot_direct_us"] / 1e3,
-                                             blk["breakdown"], c["kernels_loaded"], blk["launches"])
+             "py_ms": ([round(pyc["median_us"] / 1e3, 3), round(pyc["p90_us"] / 1e3, 3), pyc["n"]]
+                       if pyc else None)})
+        for m, blk in configs_detail.items():
+            c = blk["cold"]
+            headline[m] = headline_entry(c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"],
+                                         blk["hot_graph_us"] / 1e3, blk["hot_direct_us"] / 1e3,
+                                         blk["breakdown"], c["kernels_loaded"], blk["launches"])
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
