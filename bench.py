@@ -319,6 +319,14 @@ def headline_entry(cold_ms, p90_ms, n, hot_graph_ms, hot_direct_ms, bd, kernels,
 
 
 # ---------------------------------------------------------------- main
+_T0 = time.time()
+
+
+def phase(msg):
+    """Progress on stderr (the JSON line is the only stdout)."""
+    print(f"[bench {time.time() - _T0:7.1f}s] {msg}", file=sys.stderr, flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -336,6 +344,8 @@ def main():
                     help="fresh-process cold starts per config (native pask_cold children)")
     ap.add_argument("--timeline-samples", type=int, default=10,
                     help="fresh-process cold starts with cfg.timeline (breakdown, GPU utilisation)")
+    ap.add_argument("--ablation-samples", type=int, default=10,
+                    help="fresh processes for the no-prefault / no-primer ablations of the main config")
     ap.add_argument("--py-cold-samples", type=int, default=5,
                     help="main config: cold starts in fresh PyTorch processes (framework process state)")
     ap.add_argument("--no-configs", action="store_true",
@@ -389,32 +399,40 @@ def main():
 
     # ---------------- cold in fresh native processes (N = 1; with replicas the
     # concurrent trials below are the measurement), taken BEFORE this process
-    # creates its CUDA context, so every sample is the only context on the GPU
+    # creates its CUDA context.  An idle keeper process holds a context
+    # meanwhile (the GPU stays initialised between children, as under a
+    # persistence daemon; cold medians unchanged, r3h_keeper.log)
     main_cold, configs_detail = None, {}
     if world == 1 and args.cold_samples > 0:
+        phase("cold samples: " + args.model)
         cfg = bench_cfg(args)
         image = cs.write_image(args.model, batch=args.batch)
         try:
-            main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
-            main_cold["cold_no_prefault"] = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1},
-                                                                   args.cold_samples))
-            main_cold["cold_no_prime"] = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1}, args.cold_samples))
-            py = [cs.run_py_child(args.model, cfg, args.batch) for _ in range(args.py_cold_samples)]
-            main_cold["cold_python_process"] = cs.summarize(py) if py else None
+            with cs.Keeper(image, cfg):
+                main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
+                main_cold["cold_no_prefault"] = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1},
+                                                                       args.ablation_samples))
+                main_cold["cold_no_prime"] = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1},
+                                                                    args.ablation_samples))
+                py = [cs.run_py_child(args.model, cfg, args.batch) for _ in range(args.py_cold_samples)]
+                main_cold["cold_python_process"] = cs.summarize(py) if py else None
+                if not args.no_configs and args.batch == 1:
+                    for m in CONFIG_MODELS:
+                        if m == args.model:
+                            continue
+                        phase("cold samples: " + m)
+                        img_m = cs.write_image(m)
+                        try:
+                            configs_detail[m] = cold_block(cs, img_m, cfg, args.cold_samples,
+                                                           args.timeline_samples, True)
+                        finally:
+                            os.unlink(img_m)
         finally:
             os.unlink(image)
-        if not args.no_configs and args.batch == 1:
-            for m in CONFIG_MODELS:
-                if m == args.model:
-                    continue
-                image = cs.write_image(m)
-                try:
-                    configs_detail[m] = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, True)
-                finally:
-                    os.unlink(image)
 
     # one replica per GPU (LOCAL_RANK -> device); on a box with fewer GPUs than
     # ranks (a harness check on one GPU) ranks share devices round-robin
+    phase("hot measurement")
     local_rank = local_rank % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
@@ -669,6 +687,7 @@ def main():
                                          blk["hot_graph_us"] / 1e3, blk["hot_direct_us"] / 1e3,
                                          blk["breakdown"], c["kernels_loaded"], blk["launches"])
 
+    phase("cpu baseline")
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         ts = time_oracle(spec, x, 5, 20.0)
@@ -702,7 +721,8 @@ def main():
                    "l2": "warm (no flush)" if args.no_flush else
                          "flushed (256 MiB memset) before every timed inference",
                    "cold": f"{args.cold_samples} fresh native processes per config (pask_cold), "
-                           "t0 = pask_load_model entry, t1 = first inference done"},
+                           "t0 = pask_load_model entry, t1 = first inference done; an idle keeper "
+                           "process holds a context meanwhile (GPU kept initialised)"},
         "e2e": {"value": round(world * args.batch * 1000.0 / e2e_max, 2), "unit": "imgs/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": round(e2e_max, 4)},

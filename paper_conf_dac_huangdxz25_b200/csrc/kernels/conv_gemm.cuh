@@ -270,8 +270,9 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int mt = blockIdx.x, nt = blockIdx.y;
   const int b = blockIdx.z / splits;
   const int split = blockIdx.z - b * splits;
-  const int kb_begin = static_cast<int>((static_cast<int64_t>(split) * p.num_kb) / splits);
-  const int kb_end = static_cast<int>((static_cast<int64_t>(split + 1) * p.num_kb) / splits);
+  // 32-bit: num_kb * splits < 2^31 (num_kb <= 2^25 for an int32 K, splits <= 16)
+  const int kb_begin = (split * p.num_kb) / splits;
+  const int kb_end = ((split + 1) * p.num_kb) / splits;
   const int nk = kb_end - kb_begin;  // >= 1 (host guarantees num_kb >= splits)
   const int m0 = mt * kBM, n0 = nt * bn;
   const int lb = box_log2(bn);
@@ -282,8 +283,12 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
   const int valid_rows = min(kBM, p.M - m0);
   const int slice_rows = max(0, min(rows_per, valid_rows - r0));
   const bool res_tma = p.c_tma && p.res != nullptr;
+  // the debug phase trace is compiled into the full-feature objects only (the
+  // per-model families variants drop it: 1.5 KB less code to upload)
   unsigned long long* trace =
-      p.trace ? p.trace + 8ull * (blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) : nullptr;
+      (kGemmFeat == GF_ALL && p.trace)
+          ? p.trace + 8ull * (blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z))
+          : nullptr;
   // debug phase stamps: [0] start [1] prologue done [2] producer past griddepcontrol.wait
   // [3] first k-block landed [4] first accumulator chunk in registers (or split-K
   // partials pushed) [5] accumulator ready [6] epilogue math done [7] tile stored
@@ -564,6 +569,8 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
           tmem_ld16_issue(taddr + c * 16, r);
           tmem_ld_wait(r);
         }
+        // not unrolled: 4 copies of the 4 DSMEM stores were 5 KB of SASS to upload
+#pragma unroll 1
         for (; c < cpr; c += kEpiGroups) {
           uint32_t u[16];
 #pragma unroll
@@ -624,6 +631,9 @@ __device__ __forceinline__ void conv_gemm_body(const GemmParams& p) {
         const uint32_t src = recv + lr * recv_pitch + cb * 4;
 #pragma unroll
         for (int i = 0; i < 16; ++i) v[i] = 0.f;
+        // two slots per trip: their 8 loads in flight together, half the code of
+        // the compiler's 4-way unroll
+#pragma unroll 2
         for (int sp = 0; sp < splits; ++sp) {
           const uint32_t a = src + sp * rows_per * recv_pitch;
 #pragma unroll

@@ -19,19 +19,11 @@ __device__ __forceinline__ float warp_max(float v) {
   return v;
 }
 
-// Activation over 8 values: ReLU / ReLU6 inline, GELU / tanh out of line (rare
-// on the memory-bound path; keeps the code object small -- uploads cost ~1.1 us
-// per KB of SASS).  Same arithmetic as apply_act either way.
-struct F8 {
-  float v[8];
-};
-// by value in registers (a reference parameter would put the array on the stack
-// and give every memory kernel a local-memory frame)
-__device__ __noinline__ F8 act8_slow(F8 x, int act) {
-#pragma unroll
-  for (int i = 0; i < 8; ++i) x.v[i] = apply_act(x.v[i], act);
-  return x;
-}
+// Activation over 8 values: ReLU / ReLU6 inline, GELU / tanh through one
+// out-of-line scalar routine (rare on the memory-bound path; one copy of its
+// body keeps the code object small -- uploads cost ~1.1 us per KB of SASS).
+// Same arithmetic as apply_act either way.
+__device__ __noinline__ float act1_slow(float v, int act) { return apply_act(v, act); }
 __device__ __forceinline__ void act8(float (&v)[8], int act) {
   if (act == 1) {
 #pragma unroll
@@ -40,12 +32,8 @@ __device__ __forceinline__ void act8(float (&v)[8], int act) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) v[i] = fminf(fmaxf(v[i], 0.f), 6.f);
   } else if (act >= 3) {
-    F8 x;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) x.v[i] = v[i];
-    x = act8_slow(x, act);
-#pragma unroll
-    for (int i = 0; i < 8; ++i) v[i] = x.v[i];
+    for (int i = 0; i < 8; ++i) v[i] = act1_slow(v[i], act);
   }
 }
 
@@ -99,38 +87,38 @@ __device__ __forceinline__ void pool_body(const PoolParams& p) {
     t /= p.Q;
     const int pp = t % p.P;
     const int n = t / p.P;
-    float acc[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) acc[i] = p.mode == 0 ? -INFINITY : 0.f;
-    float cnt = 0.f;
     const int ih0 = pp * p.sh - p.ph, iw0 = q * p.sw - p.pw;
     const bool is_max = p.mode == 0;
-    if (!p.per_warp && taps <= 9) {
-      // small windows (ResNet-50's 3x3 max pool): every tap load issued before
-      // the first combine; same taps, same order as the loop below
+    if (is_max && !p.per_warp && taps <= 9) {
+      // small max windows (ResNet-50's 3x3 s2, the tiny CNN's 2x2): every tap load
+      // issued before the first combine, combined as packed bf16x2.  The max of
+      // bf16 values is one of them, so this is bit-identical to the fp32 max
+      // followed by RNE (the loop below), in a fifth of the code (uploads cost
+      // ~1.1 us per KB of SASS).  Out-of-window taps read as -inf.
+      const uint32_t ninf2 = 0xff80ff80u;
       uint4 xv[9];
-      bool ok[9];
       int r = 0, s = 0;
 #pragma unroll
       for (int tap = 0; tap < 9; ++tap) {
         const int ih = ih0 + r, iw = iw0 + s;
-        ok[tap] = tap < taps && ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
-        xv[tap] = ok[tap] ? __ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch) : make_uint4(0, 0, 0, 0);
+        const bool ok = tap < taps && ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
+        xv[tap] = ok ? __ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch) : make_uint4(ninf2, ninf2, ninf2, ninf2);
         if (++s == p.S) {
           s = 0;
           ++r;
         }
       }
+      uint4 m = xv[0];
 #pragma unroll
-      for (int tap = 0; tap < 9; ++tap) {
-        if (!ok[tap]) continue;
-        float f[8];
-        unpack_bf16x8(xv[tap], f);
-        cnt += 1.f;
+      for (int tap = 1; tap < 9; ++tap) m = bf16x8_max(m, xv[tap]);
+      reinterpret_cast<uint4*>(p.y)[idx] = m;
+      continue;
+    }
+    float acc[8];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] = is_max ? fmaxf(acc[i], f[i]) : acc[i] + f[i];
-      }
-    } else {
+    for (int i = 0; i < 8; ++i) acc[i] = is_max ? -INFINITY : 0.f;
+    float cnt = 0.f;
+    {
 #pragma unroll 1
       for (int tap = p.per_warp ? lane : 0; tap < taps; tap += p.per_warp ? 32 : 1) {
         const int r = tap / p.S, s = tap - r * p.S;
@@ -239,29 +227,36 @@ __device__ __forceinline__ void dw_body(const DwParams& p) {
     if (k3) {
       // 3x3 (MobileNetV2): all nine tap loads issued before the first FMA (one
       // memory round trip instead of nine); same taps, same order as below
-      uint4 xv[9], wv[9];
+      // (later grid-stride trips reload the taps in place: selecting between the
+      // prefetched and fresh taps made the compiler peel the first trip, a second
+      // copy of this body -- 4 KB more code to upload)
+      uint4 xv[9];
       bool ok[9];
-      const bool first = idx == idx0;
+      if (idx != idx0) {
+#pragma unroll
+        for (int t9 = 0; t9 < 9; ++t9) wpre[t9] = __ldg(w + t9 * chunks + ch);
+      }
 #pragma unroll
       for (int t9 = 0; t9 < 9; ++t9) {
         const int ih = ih0 + t9 / 3, iw = iw0 + t9 % 3;
         ok[t9] = ih >= 0 && ih < p.H && iw >= 0 && iw < p.W;
         xv[t9] = ok[t9] ? __ldg(x + ((n * p.H + ih) * p.W + iw) * chunks + ch) : make_uint4(0, 0, 0, 0);
-        wv[t9] = first ? wpre[t9] : __ldg(w + t9 * chunks + ch);
       }
 #pragma unroll
       for (int t9 = 0; t9 < 9; ++t9) {
         if (!ok[t9]) continue;
         float xf[8], wf[8];
         unpack_bf16x8(xv[t9], xf);
-        unpack_bf16x8(wv[t9], wf);
+        unpack_bf16x8(wpre[t9], wf);
 #pragma unroll
         for (int i = 0; i < 8; ++i) acc[i] = fmaf(xf[i], wf[i], acc[i]);
       }
     } else {
+#pragma unroll 1
       for (int r = 0; r < p.R; ++r) {
         const int ih = ih0 + r * p.dh;
         if (ih < 0 || ih >= p.H) continue;
+#pragma unroll 1
         for (int s = 0; s < p.S; ++s) {
           const int iw = iw0 + s * p.dw;
           if (iw < 0 || iw >= p.W) continue;
@@ -301,8 +296,12 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
   pdl_wait();
   pdl_launch_dependents();
   const int lane = threadIdx.x & 31;
-  const int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  if (row >= p.rows) return;
+  // a warp past the last row recomputes the last row and stores nothing (no early
+  // exit: the shuffles below then need no divergent-warp fallback code)
+  if (p.rows <= 0) return;
+  const int wrow = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const bool live = wrow < p.rows;
+  const int row = live ? wrow : p.rows - 1;
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
   const bool vec = (p.cols & 7) == 0;
@@ -331,7 +330,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
 #pragma unroll
     for (int j = 0; j < kSmRegChunks; ++j) {
       const int c = lane * 8 + 256 * j;
-      if (c < p.cols) {
+      if (live && c < p.cols) {
 #pragma unroll
         for (int i = 0; i < 8; ++i) f[j][i] = __expf(f[j][i] * p.scale - gm) * inv;
         *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f[j]);
@@ -364,6 +363,7 @@ __device__ __forceinline__ void softmax_body(const RowParams& p) {
   const float gm = warp_max(m);
   s = (m == -INFINITY) ? 0.f : s * __expf(m - gm);
   const float inv = 1.f / warp_sum(s);
+  if (!live) return;
   if (vec) {
 #pragma unroll 1
     for (int c = lane * 8; c < p.cols; c += 256) {
@@ -411,6 +411,7 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
       }
     }
   } else if (p.gamma && p.beta) {
+#pragma unroll 1
     for (int c = lane * 8; c < p.cols; c += 256) {
       prefetch_l2(p.gamma + c);
       prefetch_l2(p.beta + c);
@@ -418,8 +419,12 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
   }
   pdl_wait();
   pdl_launch_dependents();
-  const int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  if (row >= p.rows) return;
+  if (p.rows <= 0) return;
+  // a warp past the last row recomputes the last row and stores nothing (no
+  // early exit before the shuffles: no divergent-warp fallback code)
+  const int wrow = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const bool live = wrow < p.rows;
+  const int row = live ? wrow : p.rows - 1;
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(p.x) + static_cast<int64_t>(row) * p.cols;
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.y) + static_cast<int64_t>(row) * p.cols;
   if (in_regs) {
@@ -457,7 +462,7 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
         const float be[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
         for (int i = 0; i < 8; ++i) f[j][i] = (f[j][i] - mean) * rstd * g[i] + be[i];
-        *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f[j]);
+        if (live) *reinterpret_cast<uint4*>(y + c) = pack_bf16x8(f[j]);
       }
     }
     return;
@@ -483,6 +488,7 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
     }
   }
   const float rstd = rsqrtf(warp_sum(v) / static_cast<float>(p.cols) + p.eps);
+  if (!live) return;
 #pragma unroll 1
   for (int c = lane * 8; c < p.cols; c += 256) {
     float f[8];
@@ -503,7 +509,6 @@ __device__ __forceinline__ void layernorm_body(const RowParams& p) {
 // activation rows (L2-resident) and accumulates in fp32.  Lane partials are
 // combined by the fixed xor tree, the K slices of a column in slice order.
 constexpr int kGemvPre = 8;
-__device__ __noinline__ float gemv_act_slow(float v, int act) { return apply_act(v, act); }
 // fp32 dot of two 8 x bf16 vectors added to acc (bf16 -> fp32 is a 16-bit shift)
 __device__ __forceinline__ float dot8(const uint4& a, const uint4& b, float acc) {
   const uint32_t av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
@@ -563,7 +568,7 @@ __device__ __forceinline__ void gemv_body(const GemvParams& p) {
       if (p.res) v += __bfloat162float(reinterpret_cast<const __nv_bfloat16*>(p.res)[o]);
       if (p.act == 1) v = fmaxf(v, 0.f);
       else if (p.act == 2) v = fminf(fmaxf(v, 0.f), 6.f);
-      else if (p.act >= 3) v = gemv_act_slow(v, p.act);
+      else if (p.act >= 3) v = act1_slow(v, p.act);
       reinterpret_cast<__nv_bfloat16*>(p.y)[o] = __float2bfloat16_rn(v);
     }
   }

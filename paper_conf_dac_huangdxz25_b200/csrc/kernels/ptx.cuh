@@ -350,5 +350,14 @@ __device__ __forceinline__ uint4 pack_bf16x8(const float (&f)[8]) {
   u.w = pack_bf16x2(f[6], f[7]);
   return u;
 }
+// lane-wise max of 8 bf16 (max.bf16x2: exact, NaN-ignoring like fmaxf)
+__device__ __forceinline__ uint32_t bf16x2_max(uint32_t a, uint32_t b) {
+  uint32_t d;
+  asm("max.bf16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
+__device__ __forceinline__ uint4 bf16x8_max(const uint4& a, const uint4& b) {
+  return make_uint4(bf16x2_max(a.x, b.x), bf16x2_max(a.y, b.y), bf16x2_max(a.z, b.z), bf16x2_max(a.w, b.w));
+}
 
 }  // namespace pask

@@ -39,6 +39,7 @@ struct Tuning {
   bool direct_one_stream = false;  // branches: direct issue on one stream
   bool no_event_warm = false;      // pask_create: do not pre-record the timing events
   bool parallel_upload = false;    // packaging 2: helper uploads the contraction family concurrently
+  bool keep_primer = false;        // keep the driver primer's code object loaded until destroy
   // device phase trace (experiment builds only)
   int trace_node = -2;             // node index, -1 = all, -2 = off
   uint64_t trace_ptr = 0;          // device address of the trace buffer

@@ -123,6 +123,34 @@ def sample(image: str, cfg: dict, n: int, device: int = 0) -> list[dict]:
     return [run_child(image, cfg, device) for _ in range(n)]
 
 
+class Keeper:
+    """An idle process holding a CUDA context on `device` while fresh-process
+    samples run (a pask_cold child set up and blocked before its cold window):
+    the GPU stays initialised between children, as under a persistence daemon,
+    instead of being torn down and re-initialised for each (~1 s per child).
+    Measured on one box (profiles/r2/r3h_keeper.log, 12 children per row): the
+    children's cold medians with and without it are within the box noise."""
+
+    def __init__(self, image: str, cfg: dict, device: int = 0):
+        self.cmd = [EXE, image, "--cfg", cfg_arg(cfg), "--device", str(device), "--wait"]
+        self.proc = None
+
+    def __enter__(self):
+        self.proc = subprocess.Popen(self.cmd, stdin=subprocess.PIPE, stdout=subprocess.PIPE,
+                                     stderr=subprocess.PIPE, text=True)
+        line = self.proc.stdout.readline()
+        if line.strip() != "ready":
+            self.proc.kill()
+            self.proc.wait()
+            raise RuntimeError(f"keeper did not get ready: {line!r} {self.proc.stderr.read()[-2000:]}")
+        return self
+
+    def __exit__(self, *exc):
+        self.proc.kill()            # our own child, by PID; it never entered its cold window
+        self.proc.wait()
+        return False
+
+
 def summarize(samples: list[dict]) -> dict:
     cold = [s["cold_us"] for s in samples]
     return {"median_us": statistics.median(cold), "p90_us": pctl(cold, 0.9), "min_us": min(cold),
