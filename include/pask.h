@@ -209,7 +209,9 @@ typedef struct {
                              solution the plan binds and whose contraction entry compiles
                              every path the plan's contraction nodes take (D13);
                          3 = one CUfunction `pask_all` for both families (D10:
-                             one upload, measured slower on the hot path; not the default) */
+                             one upload for the cold start, in the same per-model variants;
+                             slower on the hot path until pask_promote repacks the model
+                             into the two family entries, D15) */
   int32_t interleave; /* 0 = load-first (default): the first inference launches once every
                          planned kernel is uploaded -- on this driver a code upload waits for
                          all running GPU work, so
@@ -365,7 +367,14 @@ int pask_infer_host(pask_ctx *ctx, const void *const *host_inputs, void *const *
  * Synchronous and meant for the gap between requests: it first waits for the
  * in-flight inference (uploads wait for running GPU work, D3).
  * Results stay within tolerance; a graph captured for hot replay is re-captured.
- * *promoted (may be NULL) = number of nodes rebound. */
+ * *promoted (may be NULL) = number of nodes rebound.
+ * Under packaging 3 the call only repacks (D15): it uploads the two
+ * family entries of the variant with the same cases and paths as the loaded
+ * single entry, moves every node served by pask_all onto them (same bodies:
+ * outputs bitwise equal) and switches the context to packaging 2 -- the cold
+ * start pays one upload, the hot path gets per-entry register allocation and
+ * the memory solutions' small parameter block; *promoted = nodes moved, the
+ * plan is unchanged.  A later call promotes as above. */
 int pask_promote(pask_ctx *ctx, int32_t target_catalog, int32_t *promoted);
 
 /* Wait for the last issued inference and finalise its timing statistics

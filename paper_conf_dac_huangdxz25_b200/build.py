@@ -76,11 +76,16 @@ FAMILY_VARIANTS = {"pask_families_tf": (0x30, 0x17), "pask_families_dwg": (0x5b,
                    "pask_families": (0x7f, 0x7f)}
 FAMILY_SOFTMAX_REG = {"pask_families_tf": 1, "pask_families_dwg": 0, "pask_families_cnn": 0,
                       "pask_families_dw": 1, "pask_families": 1}
-EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS}, "pask_single": ["pask_all"],
+# Packaging 3 comes in the same variants: pask_single_<v> has the cases and paths
+# of pask_families_<v> behind the one entry pask_all (pask_single: everything).
+SINGLE_VARIANTS = {k.replace("pask_families", "pask_single"): v for k, v in FAMILY_VARIANTS.items()}
+SINGLE_SOFTMAX_REG = {k.replace("pask_families", "pask_single"): v for k, v in FAMILY_SOFTMAX_REG.items()}
+EXTRA_OBJECTS = {**{k: ["pask_conv_igemm", "pask_mem"] for k in FAMILY_VARIANTS},
+                 **{k: ["pask_all"] for k in SINGLE_VARIANTS},
                  "pask_primer": ["pask_primer"]}   # pask_create's driver primer (not a solution)
 EXTRA_DEFINES = {k: [f"-DPASK_MEM_MASK={m:#x}", f"-DPASK_GEMM_FEAT={g:#x}",
-                     f"-DPASK_SOFTMAX_REG={FAMILY_SOFTMAX_REG[k]}"]
-                 for k, (m, g) in FAMILY_VARIANTS.items()}
+                     f"-DPASK_SOFTMAX_REG={({**FAMILY_SOFTMAX_REG, **SINGLE_SOFTMAX_REG})[k]}"]
+                 for k, (m, g) in {**FAMILY_VARIANTS, **SINGLE_VARIANTS}.items()}
 
 # The "tuned library": one specialised conv solution per distinct
 # dense-conv problem (R, S, stride, pad, dilation, input channels C) of configs
@@ -123,6 +128,9 @@ def _gen_spec_sources():
              "// smallest first",
              "#define PASK_FAMILY_VARIANTS(X) \\"] + \
         [f"  X({k}, {m:#x}, {g:#x}) \\" for k, (m, g) in FAMILY_VARIANTS.items()] + ["", ""]
+    host += ["// packaging 3 single-entry variants, the same masks, smallest first",
+             "#define PASK_SINGLE_VARIANTS(X) \\"] + \
+        [f"  X({k}, {m:#x}, {g:#x}) \\" for k, (m, g) in SINGLE_VARIANTS.items()] + ["", ""]
     for path, text in ((os.path.join(BUILD, "spec_kernels.inc"), "".join(ker)),
                        (os.path.join(BUILD, "spec_catalog.h"), "\n".join(host))):
         old = open(path).read() if os.path.exists(path) else None

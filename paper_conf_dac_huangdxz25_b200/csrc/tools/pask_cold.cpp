@@ -2,7 +2,7 @@
 // (SURVEY.md §8(d) cold protocol; the paper's cold start).
 //
 //   pask_cold MODEL.pmodel [--cfg key=value,...] [--device D] [--wait]
-//             [--sleep-ms MS] [--hot N] [--flush-mb MB] [--dump PATH]
+//             [--sleep-ms MS] [--promote] [--hot N] [--flush-mb MB] [--dump PATH]
 //
 // MODEL is a model image written by DeviceModel.save_image() (model.py): the
 // pask_graph's tensors and nodes, with every weight / bias / gamma / beta and
@@ -17,7 +17,9 @@
 //      the per-kernel load timeline and, with cfg timeline=1, the per-node GPU
 //      intervals; --hot N then times N more inferences (CUDA events, L2 flushed
 //      by a --flush-mb memset before each when MB > 0); --dump writes every
-//      tensor's bytes, in tensor order, after the cold inference.
+//      tensor's bytes, in tensor order, after the cold inference; --promote
+//      calls pask_promote (idle-interval loading; packaging 3: the repack into
+//      the two family entries, D15) before the hot inferences.
 // No PyTorch, no Python: the whole process is native, so a sample costs
 // milliseconds of process start instead of seconds of interpreter start.
 #include <dlfcn.h>
@@ -192,12 +194,13 @@ int main(int argc, char** argv) {
   if (argc < 2) {
     fprintf(stderr,
             "usage: pask_cold MODEL.pmodel [--cfg k=v,...] [--device D] [--wait] [--sleep-ms MS] "
-            "[--hot N] [--flush-mb MB] [--dump PATH]\n");
+            "[--promote] [--hot N] [--flush-mb MB] [--dump PATH]\n");
     return 1;
   }
   const char* model = argv[1];
   pask_config cfg{1, 0, 0, 2, 1, 0, 0, 0, 0, 0, 0, 0, 0, 0};  // the library defaults (pask.h)
   int device = 0, hot = 0, flush_mb = 256, warm_heap_mb = 0;
+  bool promote = false;
   bool wait = false, plan_only = false, bg_spin = false, cudart = false;
   double sleep_ms = 50, spin_ms = 0;
   const char* dump = nullptr;
@@ -237,6 +240,8 @@ int main(int argc, char** argv) {
     } else if (a == "--spin-ms") {  // busy-wait (core kept awake) instead of sleeping before t0
       spin_ms = atof(next());
       sleep_ms = 0;
+    } else if (a == "--promote") {
+      promote = true;
     } else if (a == "--hot") {
       hot = atoi(next());
     } else if (a == "--flush-mb") {
@@ -491,6 +496,11 @@ int main(int argc, char** argv) {
       fwrite(h.data(), 1, h.size(), f);
     }
     fclose(f);
+  }
+  if (promote) {
+    int32_t n = 0;
+    pk(pask_promote(pc, -1, &n), "pask_promote");
+    kv("promoted", n);
   }
   if (hot > 0) {  // hot inferences in the same process (CUDA events on the stream)
     CUevent e0, e1;

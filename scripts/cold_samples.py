@@ -63,8 +63,16 @@ def write_image(model: str, path: str | None = None, batch: int = 1) -> str:
 
 
 def run_child(image: str, cfg: dict, device: int = 0, hot: int = 0, dump: str | None = None,
-              flush_mb: int = 256, timeout: float = 120.0, env: dict | None = None) -> dict:
+              flush_mb: int = 256, timeout: float = 120.0, env: dict | None = None,
+              promote: bool | None = None) -> dict:
+    """One fresh native process.  promote (default: with hot inferences under
+    packaging 3) calls pask_promote after the cold inference -- the idle-interval
+    repack into the two family entries (D15) -- before the hot ones."""
     cmd = [EXE, image, "--cfg", cfg_arg(cfg), "--device", str(device)]
+    if promote is None:
+        promote = bool(hot) and cfg.get("packaging") == 3
+    if promote:
+        cmd += ["--promote"]
     if hot:
         cmd += ["--hot", str(hot), "--flush-mb", str(flush_mb)]
     if dump:

@@ -168,6 +168,38 @@ def test_single_function_packaging_bitwise(name):
 
 
 @pytest.mark.parametrize("name", MODELS)
+def test_single_function_repack_bitwise(name):
+    """Packaging 3 then pask_promote (D15): the cold inference runs on
+    the single entry (one upload); the idle-interval repack uploads the two
+    family entries of the variant with the same masks and re-lowers the nodes.
+    Every later inference -- direct issue and CUDA-graph replay -- is bitwise
+    equal to the cold one, and every solution stays resident."""
+    import torch
+    spec, x = build_model(name)
+    dm, ctx, plan = run_model(spec, x, cfg=P.config(packaging=3, graph=1, branches=1))
+    cold = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
+    k0 = ctx.stats()["kernels_loaded"]
+    n = ctx.promote()
+    fam = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM, P.K_GEMV,
+           P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
+    assert n == sum(1 for b in plan if b[2] in fam)
+    bound_fams = {"mem" if b[2] in (P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX,
+                                    P.K_LAYERNORM, P.K_GEMV) else "contract" for b in plan if b[2] in fam}
+    assert ctx.stats()["kernels_loaded"] == k0 + len(bound_fams)
+    assert all(ctx.kernel_is_loaded(b[2]) for b in plan)
+    assert [tuple(b) for b in ctx.bindings()] == [tuple(b) for b in plan]
+    s = torch.cuda.current_stream().cuda_stream
+    for _ in range(3):                                   # direct, then capture + replays
+        for L in spec["layers"]:
+            dm.t[L["out"]].zero_()
+        ctx.infer(s)
+        ctx.sync()
+        for L in spec["layers"]:
+            np.testing.assert_array_equal(cold[L["out"]], dm.read_raw(L["out"]))
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", MODELS)
 def test_model_hot_repeat_bitwise(name):
     """A second (hot) inference reproduces the first bit for bit (deterministic
     split-K; no atomics in any reduction order)."""

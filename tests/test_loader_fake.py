@@ -241,9 +241,10 @@ def test_branches_issue_side_nodes_after_their_producer(name):
         assert sum(1 for _, kind in launches if kind == 3) == len(side)
 
 
+@pytest.mark.parametrize("packaging", [2, 3])
 @pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnn"), ("mobilenet_v2", "dwg"),
                                           ("bert_base", "tf"), ("bert_base_fa", "tf")])
-def test_family_variant_covers_the_plan(name, variant):
+def test_family_variant_covers_the_plan(name, variant, packaging):
     """Packaging 2 (D8): the families object is loaded in the smallest
     variant whose memory-bound cases cover every solution the plan binds (CNN:
     layout / pool / softmax / GEMV; layout / depthwise / global-average pool /
@@ -251,12 +252,13 @@ def test_family_variant_covers_the_plan(name, variant):
     plan's contraction nodes take (D13: split-K / gather / im2col for
     the CNNs, staged epilogues for MobileNetV2's N = 24 layers, MN-major B and
     GELU for BERT); one code object, whose bytes are that variant's image
-    (attention keeps its own object)."""
+    (attention keeps its own object).  Packaging 3 (D10) picks the single-entry
+    variant pask_single_<v> with the same masks: one CUfunction."""
     from paper_conf_dac_huangdxz25_b200 import build as B
     spec, _ = build_model(name)
     dm = DeviceModel(spec, alloc=False)
     P.test_fake_driver(True, load_us=0)
-    ctx = P.Context(0, P.config(packaging=2))
+    ctx = P.Context(0, P.config(packaging=packaging))
     plan = ctx.load_model(dm.graph)
     ctx.infer(0)
     ctx.sync()
@@ -272,9 +274,44 @@ def test_family_variant_covers_the_plan(name, variant):
     names = list(B.FAMILY_VARIANTS)
     assert names.index(f"pask_families_{variant}") <= names.index("pask_families_dw")
     own = [b[2] for b in plan if b[2] == P.K_ATTENTION][:1]
-    expect = os.path.getsize(os.path.join(B.BUILD, f"pask_families_{variant}.fatbin"))
+    stem = "pask_families" if packaging == 2 else "pask_single"
+    assert B.SINGLE_VARIANTS[f"pask_single_{variant}"] == B.FAMILY_VARIANTS[f"pask_families_{variant}"]
+    expect = os.path.getsize(os.path.join(B.BUILD, f"{stem}_{variant}.fatbin"))
     expect += sum(os.path.getsize(os.path.join(B.BUILD, P.kernel_name(k) + ".fatbin")) for k in own)
     assert st["code_bytes_loaded"] == expect
+    assert st["kernels_loaded"] == (2 if packaging == 2 else 1) + len(own)
+
+
+@pytest.mark.parametrize("name,variant", [("resnet50", "cnn"), ("mobilenet_v2", "dwg"), ("bert_base", "tf")])
+def test_single_entry_repack(name, variant):
+    """DESIGN.md D15: packaging 3 cold-starts on pask_single_<v> (one upload);
+    pask_promote then repacks -- uploads pask_families_<v> (the same masks; one
+    more parse, two more functions), moves every family-served node and leaves
+    the plan alone; the next inferences issue from the family entries."""
+    from paper_conf_dac_huangdxz25_b200 import build as B
+    spec, _ = build_model(name)
+    dm = DeviceModel(spec, alloc=False)
+    P.test_fake_driver(True, load_us=0)
+    ctx = P.Context(0, P.config(packaging=3, graph=1))
+    plan = ctx.load_model(dm.graph)
+    ctx.infer(0)
+    ctx.sync()
+    st0 = ctx.stats()
+    fam = {P.K_LAYOUT, P.K_CONV_DW, P.K_POOL, P.K_POOL_GAVG, P.K_SOFTMAX, P.K_LAYERNORM, P.K_GEMV,
+           P.K_CONV_IGEMM, P.K_CONV_1X1, P.K_GEMM}
+    n = ctx.promote()
+    assert n == sum(1 for b in plan if b[2] in fam)
+    st1 = ctx.stats()
+    assert st1["kernels_loaded"] == st0["kernels_loaded"] + 2
+    single = os.path.getsize(os.path.join(B.BUILD, f"pask_single_{variant}.fatbin"))
+    families = os.path.getsize(os.path.join(B.BUILD, f"pask_families_{variant}.fatbin"))
+    assert st1["code_bytes_loaded"] - st0["code_bytes_loaded"] == families
+    assert st0["code_bytes_loaded"] >= single
+    assert all(ctx.kernel_is_loaded(b[2]) for b in plan)
+    for _ in range(3):                       # direct issue, capture, replay
+        ctx.infer(0)
+        ctx.sync()
+    ctx.close()
 
 
 def test_create_refuses_a_context_of_another_device():
