@@ -324,8 +324,12 @@ int pask_create(pask_ctx **ctx, int device, const pask_config *cfg);
 int pask_plan(const pask_graph *g, const pask_config *cfg, pask_binding *plan_out,
               pask_stats_t *stats_out);
 
-/* Bytes of zero-filled device workspace the graph needs (split-K partials and
- * tile counters); host-only. */
+/* Bytes of device workspace the graph needs; host-only, a pure function of the
+ * graph's shapes (and the PASK_STEM_FOLD switch).  Today: the stem fold of
+ * DESIGN.md D16 -- a conv fed by a layout node over few input channels (the
+ * ResNet-50 7x7 s2 stem) reads a regrouped copy of its input and weights that
+ * the layout kernel writes here each inference.  0 when no node needs any.
+ * pask_load_model fails with PASK_ENOMEM if g->workspace is null or smaller. */
 int pask_workspace_bytes(const pask_graph *g, uint64_t *bytes);
 
 /* Plan g (Algorithm 1), then load the bound kernels in first-use order while

@@ -89,6 +89,23 @@ struct alignas(16) LayoutParams {
   void* y;         // NHWC bf16, c_out channels (c_out % 8 == 0)
   int32_t n, c, h, w, c_out;
   unsigned long long* tl;  // pask_config.timeline slots (null = off)
+  // Stem fold (D16; null yf = off; persistent CTAs over n * fT rows): the consuming conv (R x S, stride
+  // fsh x fsw, pad fph / fpw, P x Q output) is re-expressed as an fR2 x 1
+  // stride-1 conv over 64 channels, which the contraction kernel loads by TMA
+  // im2col.  Also written, from the same input:
+  //   yf[n][t][q][j*S*c + s*c + ci] = x[n][ci][fsh*t - fph + j][fsw*q - fpw + s]
+  //     (0 outside the image and for channels >= fsh*S*c),  t < fT = P + fR2 - 1
+  //   wf[k][r2][j*S*c + s*c + ci]   = wsrc[k][fsh*r2 + j][s][ci]  (KRSC, fcw channels;
+  //     0 where fsh*r2 + j >= R or the channel is padding)
+  void* yf;              // bf16 [n][fT][fQ][64] (workspace)
+  const void* wsrc;      // bf16 [fK][fR][fS][fcw], the conv's weights; null: wf already
+                         // written (the first inference writes it, later ones skip it)
+  void* wf;              // bf16 [fK][fR2][64] (workspace)
+  int32_t fT, fQ, fsh, fsw, fph, fpw, fR, fS, fR2, fK, fcw;
+  int32_t fWp;           // smem row pitch of the staged input rows
+  int32_t frow_ctas;     // CTAs [0, frow_ctas) walk the folded rows; the rest write wf
+  uint16_t foff[64];     // smem element offset of folded channel cc in a staged row
+                         // buffer ((j*c + ci) * fWp + s), 0xffff for a padding channel
 };
 
 struct alignas(16) PoolParams {

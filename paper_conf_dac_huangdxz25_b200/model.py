@@ -227,6 +227,9 @@ class DeviceModel:
         if self.alloc and self.ws_bytes:
             self.ws = torch.zeros(self.ws_bytes, dtype=torch.uint8, device=self.device)
             self._make_graph(self.ws.data_ptr(), self.ws_bytes)
+        elif self.ws_bytes:  # host-only graph: a placeholder range like every tensor's
+            self.ws = None
+            self._make_graph(self._fake(self.ws_bytes), self.ws_bytes)
         else:
             self.ws = None
 

@@ -177,8 +177,18 @@ def test_catalog_introspection_and_workspace():
     assert lib.pask_num_kernels() == len(OP.KERNEL_NAMES) == P.NUM_KERNELS + len(OP.SPECS)
     assert [P.kernel_name(k) for k in range(P.num_kernels())] == OP.KERNEL_NAMES
     assert P.kernel_name(99) == ""
-    spec, _ = build_model("resnet50")
-    assert P.workspace_bytes(DeviceModel(spec, alloc=False).graph) == 0
+    # the only workspace is the stem fold (D16): ResNet-50's 7x7 s2
+    # C = 3 stem reads Y [n][P + R2 - 1][Q][64] and weights [K][R2][64], R2 = 4;
+    # MobileNetV2's 3x3 s2 stem and the tiny CNN's 3x3 s1 conv would not take
+    # fewer k-blocks folded (2 vs 2, 3 vs 2), BERT has no conv
+    al = lambda b: (b + 255) // 256 * 256
+    for batch in (1, 3):
+        spec, _ = build_model("resnet50", batch=batch)
+        assert P.workspace_bytes(DeviceModel(spec, alloc=False).graph) == \
+            al(batch * (112 + 3) * 112 * 64 * 2) + al(64 * 4 * 64 * 2)
+    for name in ("mobilenet_v2", "tiny_cnn", "bert_base"):
+        spec, _ = build_model(name)
+        assert P.workspace_bytes(DeviceModel(spec, alloc=False).graph) == 0, name
 
 
 @pytest.mark.skipif(os.path.exists("/dev/nvidia0"), reason="GPU present")

@@ -89,6 +89,61 @@ def test_conv_gather_fallback():
     assert r.returncode == 0 and "gather ok" in r.stdout, r.stderr[-3000:]
 
 
+# Stem fold (D16): convs fed by the layout node over few channels are
+# re-expressed as R2 x 1 convs over a 64-channel regrouped input (TMA im2col).
+# (C, K, H, W, R, stride, pad, batch, act, res)
+STEM_FOLD_CASES = [
+    (3, 64, 37, 37, 7, 2, 3, 1, "relu", False),    # ResNet-50 stem geometry, ragged M
+    (3, 48, 29, 41, 7, 2, 3, 1, "none", True),     # non-square, N tail, residual (two folded-input convs)
+    (4, 32, 20, 20, 5, 2, 2, 1, "relu6", False),   # R = 5 not a multiple of the stride
+    (2, 16, 40, 33, 5, 3, 2, 1, "relu", False),    # stride 3: three rows per folded row
+    (3, 64, 224, 224, 7, 2, 3, 2, "relu", False),  # the stem at batch 2: persistent tiles
+]
+
+
+@pytest.mark.parametrize("case", STEM_FOLD_CASES, ids=[str(c) for c in STEM_FOLD_CASES])
+def test_stem_fold(case):
+    c, k, h, w, r, st, pd, n, act, res = case
+    b = _Builder("fold", 12)
+    x = b.input((n, c, h, w), "f32")
+    t = b.layout(x)
+    rr = b.conv(t, k, r, st, pd, act="none") if res else None
+    y = b.conv(t, k, r, st, pd, act=act, res=rr)
+    b.outputs = [y]
+    spec = b.spec()
+    from paper_conf_dac_huangdxz25_b200.model import DeviceModel
+    assert DeviceModel(spec, alloc=False).ws_bytes > 0, "fold not taken"
+    _check_spec(spec)
+
+
+_NOFOLD_CHILD = r"""
+import sys
+sys.path.insert(0, sys.argv[1])
+from tests.test_gpu_kernels import STEM_FOLD_CASES, _check_spec
+from tests.gpu_harness import TOL, run_model, teacher_forced_errors
+from workloads import build_model
+from paper_conf_dac_huangdxz25_b200.model import DeviceModel
+spec, x = build_model("resnet50")
+assert DeviceModel(spec, alloc=False).ws_bytes == 0
+dm, ctx, plan = run_model(spec, x)
+errs = teacher_forced_errors(dm, spec, x)
+ctx.close()
+assert max(e for _, _, e in errs) <= TOL, errs
+print("nofold ok")
+"""
+
+
+def test_resnet50_stem_unfolded():
+    """PASK_STEM_FOLD=0: ResNet-50 with its stem on the cp.async gather path."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _NOFOLD_CHILD, root], env={**os.environ, "PASK_STEM_FOLD": "0"},
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and "nofold ok" in r.stdout, r.stderr[-3000:]
+
+
 @pytest.mark.parametrize("s,hw", [(1, 56), (2, 56), (1, 7), (2, 15)])
 def test_depthwise(s, hw):
     for c in (32, 144, 960):

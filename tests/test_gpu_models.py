@@ -1,6 +1,10 @@
 """T3/T5 on the GPU: every layer of every config, teacher-forced vs the oracle,
 through the C ABI (pask_load_model -> pask_infer), plus plan / loaded-kernel
 bit-exactness against the plan oracle and cuFuncIsLoaded."""
+import os
+import subprocess
+import sys
+
 import numpy as np
 import pytest
 
@@ -77,6 +81,17 @@ def test_tuned_catalog_specialised_kernels(name):
     assert {k for k in range(P.num_kernels()) if ctx.kernel_is_loaded(k)} == set(o["loaded"])
     tuned = {L["out"]: dm.read_raw(L["out"]) for L in spec["layers"]}
     ctx.close()
+    if dm.ws_bytes and os.environ.get("PASK_STEM_FOLD") != "0":
+        # the generic solutions fold ResNet-50's stem (D16: another k
+        # order), the specialised one cannot: compare with the fold off, in a
+        # child (the runtime reads its switches once per process)
+        root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+        r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-p", "no:cacheprovider",
+                            f"{os.path.abspath(__file__)}::test_tuned_catalog_specialised_kernels[{name}]"],
+                           cwd=root, env={**os.environ, "PASK_STEM_FOLD": "0"}, capture_output=True, text=True,
+                           timeout=900)
+        assert r.returncode == 0, r.stdout[-3000:]
+        return
     dm2, ctx2, _ = run_model(spec, x)
     for L in spec["layers"]:
         np.testing.assert_array_equal(tuned[L["out"]], dm2.read_raw(L["out"]))
@@ -244,8 +259,16 @@ def test_promote_idle_interval(name):
     assert n > 0 and all(ctx.kernel_is_loaded(k) for k in o["loaded"])
     ctx.infer(stream)
     ctx.sync()
-    for L in spec["layers"]:
-        np.testing.assert_array_equal(after[L["out"]], dm.read_raw(L["out"]))
+    if dm.ws_bytes:
+        # ResNet-50's stem was folded (D16: another k order); its
+        # specialised solution runs it unfolded, so from the stem on the outputs
+        # are compared with the oracle (the unfolded bitwise check is
+        # test_tuned_catalog_specialised_kernels under PASK_STEM_FOLD=0)
+        errs = teacher_forced_errors(dm, spec, x)
+        assert max(e for _, _, e in errs) <= TOL
+    else:
+        for L in spec["layers"]:
+            np.testing.assert_array_equal(after[L["out"]], dm.read_raw(L["out"]))
     ctx.close()
 
 

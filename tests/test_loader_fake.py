@@ -242,7 +242,7 @@ def test_branches_issue_side_nodes_after_their_producer(name):
 
 
 @pytest.mark.parametrize("packaging", [2, 3])
-@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnn"), ("mobilenet_v2", "dwg"),
+@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnnf"), ("mobilenet_v2", "dwg"),
                                           ("bert_base", "tf"), ("bert_base_fa", "tf")])
 def test_family_variant_covers_the_plan(name, variant, packaging):
     """Packaging 2 (D8): the families object is loaded in the smallest
@@ -250,7 +250,7 @@ def test_family_variant_covers_the_plan(name, variant, packaging):
     layout / pool / softmax / GEMV; layout / depthwise / global-average pool /
     softmax / GEMV for MobileNetV2; softmax / LayerNorm for BERT) and whose contraction entry compiles the paths the
     plan's contraction nodes take (D13: split-K / gather / im2col for
-    the CNNs, staged epilogues for MobileNetV2's N = 24 layers, MN-major B and
+    the CNNs -- ResNet-50, its stem folded (D16), no gather --, staged epilogues for MobileNetV2's N = 24 layers, MN-major B and
     GELU for BERT); one code object, whose bytes are that variant's image
     (attention keeps its own object).  Packaging 3 (D10) picks the single-entry
     variant pask_single_<v> with the same masks: one CUfunction."""
@@ -282,7 +282,7 @@ def test_family_variant_covers_the_plan(name, variant, packaging):
     assert st["kernels_loaded"] == (2 if packaging == 2 else 1) + len(own)
 
 
-@pytest.mark.parametrize("name,variant", [("resnet50", "cnn"), ("mobilenet_v2", "dwg"), ("bert_base", "tf")])
+@pytest.mark.parametrize("name,variant", [("resnet50", "cnnf"), ("mobilenet_v2", "dwg"), ("bert_base", "tf")])
 def test_single_entry_repack(name, variant):
     """DESIGN.md D15: packaging 3 cold-starts on pask_single_<v> (one upload);
     pask_promote then repacks -- uploads pask_families_<v> (the same masks; one
@@ -352,7 +352,7 @@ def test_overlapping_tensors_run_on_one_stream():
     # a graph that aliases from the start
     dm2 = DeviceModel(spec, alloc=False)
     dm2._tensors[dm2.index[spec["layers"][5]["out"]]].dptr = dm2._tensors[dm2.index[spec["layers"][1]["out"]]].dptr
-    dm2._make_graph(None, 0)
+    dm2._make_graph(dm2.graph.workspace, dm2.ws_bytes)
     P.test_fake_driver(True)
     ctx = P.Context(0, P.config(branches=1))
     ctx.load_model(dm2.graph)
