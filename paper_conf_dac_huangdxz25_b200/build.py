@@ -60,7 +60,7 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # entry `pask_mem` in ONE code object.  name -> entries compiled into it.
 # The families object comes in variants by the memory cases compiled in
 # (PASK_MEM_MASK, bit per MemKind: layout 0, dw 1, pool 2, gavg 3, softmax 4,
-# LayerNorm 5, GEMV 6); the runtime loads the smallest covering the model's solutions
+# LayerNorm 5, GEMV 6; bit 7 the layout's stem-fold path); the runtime loads the smallest covering the model's solutions
 # (dwg = depthwise + global pool without the windowed pool: MobileNetV2).
 # Packaging 3 (D10): both families behind the single entry `pask_all`.
 # Each variant also compiles only some contraction paths (PASK_GEMM_FEAT, bit per
@@ -71,11 +71,13 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # The CNN variants also drop softmax's register-resident row path (their one
 # softmax row of 10 / 1000 classes takes the two-pass loop: same arithmetic,
 # bitwise equal) -- PASK_SOFTMAX_REG.
-FAMILY_VARIANTS = {"pask_families_tf": (0x30, 0x17), "pask_families_cnnf": (0x55, 0x41),
+FAMILY_VARIANTS = {"pask_families_tf": (0x30, 0x17), "pask_families_cnnf": (0xd5, 0x41),
                    "pask_families_dwg": (0x5b, 0x25),
                    "pask_families_cnn": (0x55, 0x61), "pask_families_dw": (0x5f, 0x7f),
-                   "pask_families": (0x7f, 0x7f)}
-# (cnnf: a CNN whose narrow stem is folded (D16) takes no cp.async gather: ResNet-50)
+                   "pask_families": (0xff, 0x7f)}
+# (cnnf: a CNN whose narrow stem is folded (D16): the layout's fold path, memory
+# bit 7, and no cp.async gather -- ResNet-50; only cnnf and the full variant
+# carry the fold path)
 FAMILY_SOFTMAX_REG = {"pask_families_tf": 1, "pask_families_cnnf": 0, "pask_families_dwg": 0,
                       "pask_families_cnn": 0, "pask_families_dw": 1, "pask_families": 1}
 # Packaging 3 comes in the same variants: pask_single_<v> has the cases and paths

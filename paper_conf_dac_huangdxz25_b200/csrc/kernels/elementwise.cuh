@@ -41,9 +41,15 @@ __device__ __forceinline__ void act8(float (&v)[8], int act) {
 // NCHW fp32 -> NHWC bf16 (RNE), channels c..c_out-1 zero.  One thread per
 // (pixel, 8-channel chunk): coalesced fp32 reads across pixels, one 16 B store.
 __device__ __noinline__ void layout_fold(const LayoutParams& p);
+#ifndef PASK_MEM_MASK
+#define PASK_MEM_MASK 0xff
+#endif
 __device__ __forceinline__ void layout_body(const LayoutParams& p) {
-  if (p.yf) {
-    layout_fold(p);
+  if (p.yf) {  // stem fold (D16): compiled into the variants whose mask has MEM_FOLD_BIT
+    if ((PASK_MEM_MASK >> MEM_FOLD_BIT) & 1)
+      layout_fold(p);
+    else
+      __trap();
     return;
   }
   pdl_wait();
@@ -101,37 +107,40 @@ __device__ __noinline__ void layout_fold(const LayoutParams& pp) {
   const float* __restrict__ x = pp.x;
   uint4* const y = static_cast<uint4*>(pp.y);
   uint4* const yf = static_cast<uint4*>(pp.yf);
-  const int C = pp.c, H = pp.h, W = pp.w, chunks = pp.c_out >> 3;
+  const int C = pp.c, H = pp.h, W = pp.w;  // host: W % 4 == 0, c_out == 8 (one NHWC chunk)
   const int fT = pp.fT, fQ = pp.fQ, fsh = pp.fsh, fsw = pp.fsw, fph = pp.fph, fpw = pp.fpw;
   const int Wp = pp.fWp, hw = H * W;
-  const int cw = pp.fS * C, used = fsh * cw;  // folded channels holding data (<= 64)
   const int tid = threadIdx.x, bd = blockDim.x;
   const int stage = fsh * C * Wp;  // elements per staging buffer
   const uint32_t s0 = smem_u32(smem_raw);
   pdl_wait();
   pdl_launch_dependents();
-  if (static_cast<int>(blockIdx.x) >= pp.frow_ctas) {  // regrouped weights (k, r2, chunk), 16 B per thread
-    const uint16_t* w = static_cast<const uint16_t*>(pp.wsrc);
-    const int fR = pp.fR, fS = pp.fS, fR2 = pp.fR2, fcw = pp.fcw;
+  if (static_cast<int>(blockIdx.x) >= pp.frow_ctas) {
+    // regrouped weights (k, r2, chunk), 16 B per thread; host tables give each
+    // folded channel's source offset within a (k, sh*r2) filter block and its j
     const int wi = (blockIdx.x - pp.frow_ctas) * bd + tid;
-    if (wi < pp.fK * fR2 * 8) {
-      const int c0 = (wi & 7) * 8, r2 = (wi >> 3) % fR2, k = (wi >> 3) / fR2;
-      uint16_t v[8];
-#pragma unroll
+    if (wi < pp.fK * pp.fR2 * 8) {
+      const int r2 = (wi >> 3) % pp.fR2, k = (wi >> 3) / pp.fR2;
+      const int blk = pp.fS * pp.fcw;
+      const uint16_t* w = static_cast<const uint16_t*>(pp.wsrc) + (k * pp.fR + fsh * r2) * blk;
+      uint64_t lo = 0, hi = 0;
+#pragma unroll 1
       for (int e2 = 0; e2 < 8; ++e2) {
-        const int cc = c0 + e2, j = cc / cw, sx = (cc - j * cw) / C, ci = cc - j * cw - sx * C;
-        const int r = fsh * r2 + j;
-        v[e2] = (cc < used && r < fR) ? w[((k * fR + r) * fS + sx) * fcw + ci] : uint16_t(0);
+        const int cc = (wi & 7) * 8 + e2, j = pp.fwj[cc];
+        const uint64_t v = (j != 0xff && fsh * r2 + j < pp.fR) ? w[pp.fwoff[cc]] : 0;
+        if (e2 < 4) lo |= v << (16 * e2); else hi |= v << (16 * (e2 - 4));
       }
-      reinterpret_cast<uint4*>(pp.wf)[wi] = pack_u16x8(v);
+      reinterpret_cast<uint4*>(pp.wf)[wi] =
+          make_uint4(static_cast<uint32_t>(lo), static_cast<uint32_t>(lo >> 32), static_cast<uint32_t>(hi),
+                     static_cast<uint32_t>(hi >> 32));
     }
     return;
   }
+#pragma unroll 1
   for (int i = tid; i < 2 * stage; i += bd) sts_u16(s0 + 2 * i, 0);  // padding columns stay zero
   // this thread's input items (4 columns of one (j, c) row), the same every row
-  const int w4n = (W + 3) >> 2, items = fsh * C * w4n;
-  const bool vec = (W & 3) == 0;
-  int it_j[kFoldItems], it_src[kFoldItems], it_dst[kFoldItems], it_w0[kFoldItems];
+  const int w4n = W >> 2, items = fsh * C * w4n;
+  int it_j[kFoldItems], it_src[kFoldItems], it_dst[kFoldItems];
 #pragma unroll
   for (int u = 0; u < kFoldItems; ++u) {
     const int it = tid + u * bd;
@@ -140,30 +149,7 @@ __device__ __noinline__ void layout_fold(const LayoutParams& pp) {
     it_j[u] = it < items ? j : -(1 << 20);  // out of every image row: never loaded or stored
     it_src[u] = ci * hw + w0;
     it_dst[u] = 2 * (row * Wp + fpw + w0);
-    it_w0[u] = w0;
   }
-  const int nrow = pp.n * fT;
-  float4 pf[kFoldItems];
-  auto fetch = [&](int r) {
-    const int t = r % fT, n = r / fT;
-    const float* xn = x + n * C * hw;
-#pragma unroll
-    for (int u = 0; u < kFoldItems; ++u) {
-      const int hh = fsh * t - fph + it_j[u];
-      const float* src = xn + it_src[u] + hh * W;
-      pf[u] = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (hh >= 0 && hh < H) {
-        if (vec) {
-          pf[u] = __ldg(reinterpret_cast<const float4*>(src));
-        } else {
-          pf[u].x = __ldg(src);
-          if (it_w0[u] + 1 < W) pf[u].y = __ldg(src + 1);
-          if (it_w0[u] + 2 < W) pf[u].z = __ldg(src + 2);
-          if (it_w0[u] + 3 < W) pf[u].w = __ldg(src + 3);
-        }
-      }
-    }
-  };
   // the Y chunk of this thread (blockDim % 8 == 0): smem byte offsets of its 8
   // folded channels and a mask zeroing the padding channels (branch-free reads:
   // a padding channel reads offset 0 and masks it)
@@ -174,53 +160,60 @@ __device__ __noinline__ void layout_fold(const LayoutParams& pp) {
     off[e2] = o == 0xffffu ? 0u : 2u * o;
     msk |= (o == 0xffffu ? 0u : 1u) << e2;
   }
-  const int rstep = pp.frow_ctas;
-  if (static_cast<int>(blockIdx.x) < nrow) fetch(blockIdx.x);
+  const int nrow = pp.n * fT, rstep = pp.frow_ctas;
   __syncthreads();  // zero fill done
-  int buf = 0;
-  for (int r = blockIdx.x; r < nrow; r += rstep, buf ^= 1) {
-    const uint32_t sb = s0 + 2u * static_cast<uint32_t>(buf * stage);
+  // skewed pipeline, one barrier per row: iteration i issues row r_i's loads,
+  // writes row r_(i-1) out of buffer (i-1)&1 while they fly, then stages r_i in
+  // buffer i&1.  A buffer is restaged two iterations after it was staged, behind
+  // the barrier that ends the iteration which read it.
+  for (int i = 0, r = blockIdx.x;; ++i, r += rstep) {
+    float4 pf[kFoldItems];
+    const int t = r % fT, n = r / fT;
 #pragma unroll
     for (int u = 0; u < kFoldItems; ++u) {
-      if (it_j[u] >= 0) {
-        const uint32_t d = sb + it_dst[u];
-        sts_u16(d, bf16_bits(pf[u].x));
-        if (it_w0[u] + 1 < W) sts_u16(d + 2, bf16_bits(pf[u].y));
-        if (it_w0[u] + 2 < W) sts_u16(d + 4, bf16_bits(pf[u].z));
-        if (it_w0[u] + 3 < W) sts_u16(d + 6, bf16_bits(pf[u].w));
-      }
+      const int hh = fsh * t - fph + it_j[u];
+      const float* src = x + n * C * hw + it_src[u] + hh * W;
+      pf[u] = (r < nrow && hh >= 0 && hh < H) ? __ldg(reinterpret_cast<const float4*>(src))
+                                               : make_float4(0.f, 0.f, 0.f, 0.f);
     }
-    // one barrier per row: buffer buf is rewritten two rows later, after every
-    // thread has passed the next row's barrier (and so finished reading it)
-    __syncthreads();
-    if (r + rstep < nrow) fetch(r + rstep);
-    const int t = r % fT, n = r / fT;
-    // NHWC rows of this folded row (branch-free channel reads: channel
-    // min(c, C - 1), masked)
-    for (int j = 0; j < fsh; ++j) {
-      const int hh = fsh * t - fph + j;
-      if (hh < 0 || hh >= H) continue;
-      const uint32_t a = sb + 2u * static_cast<uint32_t>(j * C * Wp + fpw);
-      uint4* yo = y + static_cast<size_t>(n * H + hh) * W * chunks;
-      for (int i = tid; i < W * chunks; i += bd) {
-        const int w = chunks == 1 ? i : i / chunks, ch = i - w * chunks;
+    if (i > 0) {  // write out the previous row
+      const int rp = r - rstep, tp = rp % fT, np = rp / fT;
+      const uint32_t sb = s0 + 2u * static_cast<uint32_t>(((i - 1) & 1) * stage);
+      // NHWC rows of that folded row (branch-free channel reads: channel
+      // min(c, C - 1), masked)
+#pragma unroll 1
+      for (int j = 0; j < fsh; ++j) {
+        const int hh = fsh * tp - fph + j;
+        if (hh < 0 || hh >= H) continue;
+        const uint32_t a = sb + 2u * static_cast<uint32_t>(j * C * Wp + fpw);
+        uint4* yo = y + static_cast<size_t>(np * H + hh) * W;
+        for (int w = tid; w < W; w += bd) {
+          uint32_t v[8];
+#pragma unroll
+          for (int e2 = 0; e2 < 8; ++e2)
+            v[e2] = lds_u16(a + 2u * static_cast<uint32_t>(min(e2, C - 1) * Wp + w)) & (e2 < C ? 0xffffu : 0u);
+          yo[w] = make_uint4(v[0] | (v[1] << 16), v[2] | (v[3] << 16), v[4] | (v[5] << 16), v[6] | (v[7] << 16));
+        }
+      }
+      uint4* yrow = yf + static_cast<size_t>(rp) * fQ * 8 + (tid & 7);
+      for (int q = tid >> 3; q < fQ; q += bd >> 3) {
+        const uint32_t qo = sb + 2u * static_cast<uint32_t>(fsw * q);
         uint32_t v[8];
 #pragma unroll
-        for (int e2 = 0; e2 < 8; ++e2) {
-          const int c = ch * 8 + e2;
-          v[e2] = lds_u16(a + 2u * static_cast<uint32_t>(min(c, C - 1) * Wp + w)) & (c < C ? 0xffffu : 0u);
-        }
-        yo[i] = make_uint4(v[0] | (v[1] << 16), v[2] | (v[3] << 16), v[4] | (v[5] << 16), v[6] | (v[7] << 16));
+        for (int e2 = 0; e2 < 8; ++e2) v[e2] = lds_u16(qo + off[e2]) & ((msk >> e2) & 1u ? 0xffffu : 0u);
+        yrow[q * 8] = make_uint4(v[0] | (v[1] << 16), v[2] | (v[3] << 16), v[4] | (v[5] << 16), v[6] | (v[7] << 16));
       }
     }
-    uint4* yrow = yf + static_cast<size_t>(r) * fQ * 8 + (tid & 7);
-    for (int q = tid >> 3; q < fQ; q += bd >> 3) {
-      const uint32_t qo = sb + 2u * static_cast<uint32_t>(fsw * q);
-      uint32_t v[8];
+    if (r >= nrow) break;
+    const uint32_t sb = s0 + 2u * static_cast<uint32_t>((i & 1) * stage);
 #pragma unroll
-      for (int e2 = 0; e2 < 8; ++e2) v[e2] = lds_u16(qo + off[e2]) & ((msk >> e2) & 1u ? 0xffffu : 0u);
-      yrow[q * 8] = make_uint4(v[0] | (v[1] << 16), v[2] | (v[3] << 16), v[4] | (v[5] << 16), v[6] | (v[7] << 16));
+    for (int u = 0; u < kFoldItems; ++u) {
+      if (it_j[u] < 0) continue;
+      const float* f = &pf[u].x;
+#pragma unroll
+      for (int e2 = 0; e2 < 4; ++e2) sts_u16(sb + it_dst[u] + 2 * e2, bf16_bits(f[e2]));
     }
+    __syncthreads();
   }
 }
 

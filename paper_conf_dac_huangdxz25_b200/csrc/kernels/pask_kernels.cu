@@ -23,8 +23,9 @@ static_assert(kTimelineStride == 4096, "TimelineScope (ptx.cuh) hard-codes the e
 // CNN, CNN + depthwise, transformer) and loads the smallest one covering the
 // model's bound solutions (D8).  A case compiled out traps: the host
 // never binds it, and if it did the launch fails loudly instead of writing nothing.
+// (bit 7, MEM_FOLD_BIT: the layout's stem-fold path, D16)
 #ifndef PASK_MEM_MASK
-#define PASK_MEM_MASK 0x7f
+#define PASK_MEM_MASK 0xff
 #endif
 #define PASK_MEM_CASE(k, body) \
   case k:                     \

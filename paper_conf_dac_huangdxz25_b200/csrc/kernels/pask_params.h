@@ -106,6 +106,9 @@ struct alignas(16) LayoutParams {
   int32_t frow_ctas;     // CTAs [0, frow_ctas) walk the folded rows; the rest write wf
   uint16_t foff[64];     // smem element offset of folded channel cc in a staged row
                          // buffer ((j*c + ci) * fWp + s), 0xffff for a padding channel
+  uint16_t fwoff[64];    // weights: source offset of folded channel cc within the
+                         // (k, fsh*r2) filter rows (j*fS*fcw + s*fcw + ci)
+  uint8_t fwj[64];       // ... its j (0xff for a padding channel)
 };
 
 struct alignas(16) PoolParams {
@@ -179,6 +182,9 @@ struct alignas(16) GemvParams {
 // `pask_mem`, so one code upload makes all of them resident.  The solution's
 // own parameter block sits at offset 0; `kind` selects its body.
 enum MemKind : int32_t { MEM_LAYOUT = 0, MEM_DW, MEM_POOL, MEM_GAVG, MEM_SOFTMAX, MEM_LAYERNORM, MEM_GEMV };
+// bit of a families variant's memory mask (PASK_MEM_MASK) beyond the MemKind
+// cases: the layout kernel's stem-fold path (D16)
+constexpr int MEM_FOLD_BIT = 7;
 struct alignas(16) MemParams {
   union {
     LayoutParams l;

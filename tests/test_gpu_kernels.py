@@ -92,11 +92,12 @@ def test_conv_gather_fallback():
 # Stem fold (D16): convs fed by the layout node over few channels are
 # re-expressed as R2 x 1 convs over a 64-channel regrouped input (TMA im2col).
 # (C, K, H, W, R, stride, pad, batch, act, res)
+# (the fold needs W % 4 == 0: 16 B input loads)
 STEM_FOLD_CASES = [
-    (3, 64, 37, 37, 7, 2, 3, 1, "relu", False),    # ResNet-50 stem geometry, ragged M
-    (3, 48, 29, 41, 7, 2, 3, 1, "none", True),     # non-square, N tail, residual (two folded-input convs)
+    (3, 64, 37, 36, 7, 2, 3, 1, "relu", False),    # ResNet-50 stem geometry, odd H, ragged M
+    (3, 48, 29, 44, 7, 2, 3, 1, "none", True),     # non-square, N tail, residual (two folded-input convs)
     (4, 32, 20, 20, 5, 2, 2, 1, "relu6", False),   # R = 5 not a multiple of the stride
-    (2, 16, 40, 33, 5, 3, 2, 1, "relu", False),    # stride 3: three rows per folded row
+    (2, 16, 40, 32, 5, 3, 2, 1, "relu", False),    # stride 3: three rows per folded row
     (3, 64, 224, 224, 7, 2, 3, 2, "relu", False),  # the stem at batch 2: persistent tiles
 ]
 
