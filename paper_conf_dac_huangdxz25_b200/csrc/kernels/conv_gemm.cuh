@@ -697,10 +697,15 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
   const bool persistent = kPersistent && p.persistent != 0;
   constexpr uint32_t kABytes = kBM * kBK * 2;  // 16 KB
   const uint32_t b_bytes = static_cast<uint32_t>(bn) * kBK * 2;
-  const uint32_t stage_bytes = kABytes + b_bytes;
-  // ---- smem carve-up (mirrors gemm_tiling() on the host): ring | split-K receive
-  // slots | staging tile(s) (2 when persistent) | bias vector(s) | barriers
-  const uint32_t ring_bytes = (stages * stage_bytes + 1023u) & ~1023u;
+  // b_res (D18): a layer with one N tile keeps its whole B (every
+  // k-block of the weights) resident after the ring, loaded once per CTA; the
+  // ring then carries A only
+  const bool b_res = persistent && p.b_res != 0;
+  const uint32_t stage_bytes = kABytes + (b_res ? 0u : b_bytes);
+  // ---- smem carve-up (mirrors gemm_tiling() on the host): ring | resident B |
+  // split-K receive slots | staging tile(s) (2 when persistent) | bias vector(s) | barriers
+  const uint32_t bres_off = stages * stage_bytes;
+  const uint32_t ring_bytes = (bres_off + (b_res ? p.num_kb * b_bytes : 0u) + 1023u) & ~1023u;
   const uint32_t recv_pitch = (bn + 4) * 4;  // fp32 split-K receive row pitch (bank spread)
   const uint32_t recv_bytes = splits > 1 ? ((128u * recv_pitch + 1023u) & ~1023u) : 0u;
   const uint32_t reg0 = ring_bytes + recv_bytes;
@@ -718,6 +723,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
   const uint32_t rofree0 = smem_u32(bars + 2 * stages + 8);  // [2] staging buffer read by its store
   const uint32_t recv_bar = smem_u32(bars + 2 * stages + 10);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * stages + 11);
+  const uint32_t bres_bar = smem_u32(bars + 2 * stages + 12);  // b_res: the resident B landed
   const uint32_t ro0 = smem_base + reg0;
   const uint32_t recv = smem_base + ring_bytes;  // slot s: rows [s*rows_per, (s+1)*rows_per)
 
@@ -803,6 +809,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
       mbar_init(rofree0 + 8 * j, 1u);
     }
     mbar_init(recv_bar, 1u);
+    mbar_init(bres_bar, 1u);
     if (splits > 1) {  // the S-1 peers push the valid rows of this rank's slice, bn fp32 each
       const int sr = max(0, min(rows_per, min(kBM, p.M - mt0 * kBM) - r0));
       mbar_arrive_expect_tx(recv_bar, static_cast<uint32_t>((splits - 1) * sr * bn * 4));
@@ -855,7 +862,20 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           }
         }
         int pre = 0;
-        if (it == 0) {
+        if (it == 0 && b_res) {
+          // the resident B: every k-block once (weights before griddepcontrol.wait;
+          // an activation B, or the stem fold's first-inference weights, after it)
+          auto load_bres = [&]() {
+            mbar_arrive_expect_tx(bres_bar, static_cast<uint32_t>(nk) * b_bytes);
+#pragma unroll 1
+            for (int i = 0; i < nk; ++i)
+              tma_load_3d(smem_base + bres_off + i * b_bytes, &p.tmap_b, bres_bar, (kb_begin + i) * kBK, n0, bb);
+          };
+          if (p.b_const) load_bres();
+          pdl_wait();
+          if (!p.b_const) load_bres();
+          if (trace) trace[2] = stamp();
+        } else if (it == 0) {
           // weights of the first min(nk, stages) k-blocks before griddepcontrol.wait
           // (they overlap the previous layer's tail); ring slots start empty.  An
           // activation B operand (attention QK^T / PV) must wait like A.
@@ -882,7 +902,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           const uint32_t sa = smem_base + s * stage_bytes;
           const uint32_t sb = sa + kABytes;
           const int kb = kb_begin + i;
-          if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, b_bytes + (gather ? 0u : kABytes));
+          if (!b_done) mbar_arrive_expect_tx(full0 + 8 * s, (b_res ? 0u : b_bytes) + (gather ? 0u : kABytes));
           if (kAllowGather && im2col) {
             tma_load_im2col_4d(sa, &p.tmap_a, full0 + 8 * s, cc * 64, iw, ih, in,
                                static_cast<uint16_t>(ts * gDW), static_cast<uint16_t>(tr * gDH));
@@ -896,7 +916,7 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           } else if (!gather) {
             tma_load_3d(sa, &p.tmap_a, full0 + 8 * s, kb * kBK, m0, bb);
           }
-          if (!b_done) {
+          if (!b_done && !b_res) {
             if (p.b_major == 0) {
               tma_load_3d(sb, &p.tmap_b, full0 + 8 * s, kb * kBK, n0, bb);
             } else {
@@ -965,12 +985,13 @@ __device__ __forceinline__ void conv_gemm_body_pt(const GemmParams& p) {
           mbar_wait(tempty0 + 8 * buf, ((it >> 1) & 1) ^ 1);
           tc_fence_after();
         }
+        if (b_res && it == 0) mbar_wait(bres_bar, 0);
         for (int i = 0; i < nk; ++i) {
           mbar_wait(full0 + 8 * s, ph);
           tc_fence_after();
           if (trace && it == 0 && i == 0) trace[3] = stamp();
           const uint32_t sa = smem_base + s * stage_bytes;
-          const uint32_t sb = sa + kABytes;
+          const uint32_t sb = b_res ? smem_base + bres_off + i * b_bytes : sa + kABytes;
 #pragma unroll
           for (int k = 0; k < kBK / 16; ++k) {
             // K-major SWIZZLE_128B: +32 B per 16-element K step inside the 128 B row

@@ -82,6 +82,7 @@ struct alignas(64) GemmParams {
   uint32_t tmem_cols;  // power of two >= max(32, bn)
   uint32_t smem_bytes;
   int32_t family;      // pask_all (packaging 3): 0 = this block, 1 = the MemParams overlaid at offset 0
+  int32_t b_res;       // persistent, one N tile: B resident in smem after the ring (D18)
 };
 
 struct alignas(16) LayoutParams {

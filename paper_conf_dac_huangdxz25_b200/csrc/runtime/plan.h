@@ -62,6 +62,7 @@ struct GemmTiling {
   uint32_t smem_bytes, tmem_cols;
   int32_t persistent;  // 1: grid of min(tiles, #SMs) CTAs looping over tiles (splits == 1)
   int32_t grid_x;      // persistent grid size
+  int32_t b_res;       // persistent with one N tile: the whole B resident in smem (D18)
 };
 // Dynamic shared memory the contraction kernels may request (attribute set at load).
 constexpr uint32_t kMaxDynSmem = 220u * 1024u;

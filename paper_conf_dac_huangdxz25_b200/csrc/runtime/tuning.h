@@ -32,6 +32,7 @@ struct Tuning {
   bool no_a64 = false;        // never use 64-row A boxes
   bool no_im2col = false;     // A_GATHER instead of TMA im2col
   int stem_fold = 1;          // D16: 0 off; 1 fold a stem conv that then needs fewer k-blocks; 2 ... no more
+  bool no_b_res = false;      // D18 off: persistent one-N-tile layers stream B per k-block
   // issue / loading (pask.cpp)
   bool encode_first = false;       // proactive 2: encode, then upload (instead of concurrently)
   bool debug_cold = false;         // print per-launch host times of the cold inference
