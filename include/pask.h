@@ -268,7 +268,10 @@ typedef struct {
   uint64_t load_exposed_ns;    /* issue thread blocked on not-yet-ready kernels  */
   uint64_t issue_ns;           /* time inside cuLaunchKernelEx calls             */
   uint64_t encode_ns;          /* CUtensorMap encoding + parameter packing        */
-  uint64_t gpu_span_ns;        /* first launch -> last kernel end, last inference */
+  uint64_t gpu_span_ns;        /* first launch -> last kernel end of the last timed
+                                  inference: the first (cold) one, or every one
+                                  under timeline / instrument (a hot inference
+                                  otherwise records no timing event)            */
   uint64_t gpu_busy_ns;        /* GPU busy time of the last synced inference: the
                                   union of the kernels' [start, end] intervals
                                   (timeline = 1), or the sum of per-kernel event
@@ -354,10 +357,17 @@ int pask_load_model(pask_ctx *ctx, const pask_graph *g, pask_binding *plan_out);
  * launch (asynchronous w.r.t. the GPU). */
 int pask_infer(pask_ctx *ctx, void *const *inputs, void *const *outputs, void *cuda_stream);
 
-/* End-to-end inference from host buffers: H2D copy of every graph input from
- * host_inputs[i], pask_infer, D2H copy of every graph output into
- * host_outputs[i], then stream synchronisation.  Pinned host memory is
- * recommended; sizes follow the tensors' dims and dtype. */
+/* End-to-end inference from host buffers: every graph input from
+ * host_inputs[i], pask_infer, every graph output into host_outputs[i], then
+ * stream synchronisation; sizes follow the tensors' dims and dtype.  A pinned,
+ * device-mapped host buffer (cuMemHostAlloc / cudaHostAlloc under unified
+ * addressing) whose tensor only memory-family kernels touch (plain loads and
+ * stores: the layout / LayerNorm reading an input, the softmax / LayerNorm
+ * writing an output) is bound into the graph directly -- the kernel reads the
+ * input over the host link and writes the output there (zero copy; the launch
+ * parameters of those nodes are re-encoded on the first such call).  Any other
+ * buffer (pageable memory, or a tensor a TMA kernel touches) goes through an
+ * H2D / D2H copy into the graph's own device buffer. */
 int pask_infer_host(pask_ctx *ctx, const void *const *host_inputs, void *const *host_outputs,
                     void *cuda_stream);
 
@@ -382,7 +392,7 @@ int pask_infer_host(pask_ctx *ctx, const void *const *host_inputs, void *const *
 int pask_promote(pask_ctx *ctx, int32_t target_catalog, int32_t *promoted);
 
 /* Wait for the last issued inference and finalise its timing statistics
- * (gpu_span_ns; cold_wall_ns after the first inference). */
+ * (gpu_span_ns if it was timed; cold_wall_ns after the first inference). */
 int pask_sync(pask_ctx *ctx);
 
 /* Copy the statistics (host only; call pask_sync first for GPU times): the

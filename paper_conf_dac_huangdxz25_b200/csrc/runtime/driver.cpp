@@ -76,6 +76,7 @@ void resolve() {
   PASK_RESOLVE(cuMemFree)
   PASK_RESOLVE(cuMemsetD8)
   PASK_RESOLVE(cuMemcpyDtoH)
+  PASK_RESOLVE(cuPointerGetAttribute)
 #undef PASK_RESOLVE
   if (!all) {
     g_why = "a required CUDA driver entry point could not be resolved (driver too old?)";

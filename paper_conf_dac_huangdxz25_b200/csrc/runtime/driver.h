@@ -50,6 +50,7 @@ struct Driver {
   PASK_DRV_FN(cuMemFree)
   PASK_DRV_FN(cuMemsetD8)
   PASK_DRV_FN(cuMemcpyDtoH)
+  PASK_DRV_FN(cuPointerGetAttribute)
 #undef PASK_DRV_FN
   bool ok = false;
 };

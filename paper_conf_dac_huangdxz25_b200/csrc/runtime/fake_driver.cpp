@@ -193,6 +193,8 @@ CUresult f_event_elapsed(float* ms, CUevent, CUevent) {
 }
 CUresult f_h2d(CUdeviceptr, const void*, size_t, CUstream) { return CUDA_SUCCESS; }
 CUresult f_d2h(void*, CUdeviceptr, size_t, CUstream) { return CUDA_SUCCESS; }
+// host buffers are never device-mapped here: pask_infer_host takes the copy path
+CUresult f_ptr_attr(void*, CUpointer_attribute, CUdeviceptr) { return CUDA_ERROR_INVALID_VALUE; }
 CUresult f_stream_sync(CUstream) { return CUDA_SUCCESS; }
 // streams get handles 0x40, 0x41, ... in creation order; launches on the
 // caller's stream (0) or on the capture stream are "main" (kind 1), on any other
@@ -254,6 +256,7 @@ Driver make_fake() {
   d.cuEventElapsedTime = f_event_elapsed;
   d.cuMemcpyHtoDAsync = f_h2d;
   d.cuMemcpyDtoHAsync = f_d2h;
+  d.cuPointerGetAttribute = f_ptr_attr;
   d.cuStreamSynchronize = f_stream_sync;
   d.cuStreamCreate = f_stream_create;
   d.cuStreamDestroy = f_stream_destroy;

@@ -160,3 +160,39 @@ def test_create_binds_current_device():
         ctx = P.Context(0, P.config())
         ctx.close()
     torch.zeros(1, device="cuda").sum().item()       # torch's context still usable
+
+
+@pytest.mark.parametrize("name", ["resnet50", "bert_base"])
+def test_infer_host_zero_copy_and_copy(name):
+    """pask_infer_host (include/pask.h): pinned host buffers are bound into the
+    graph (the layout / LayerNorm reads the input over the host link, the
+    softmax / LayerNorm writes the output there), pageable ones go through
+    H2D / D2H copies; either way the output bits equal the device path's.  A
+    later pask_infer with NULL buffers is back on the graph's own device
+    buffers (the host ones are the caller's to free)."""
+    spec, x = build_model(name)
+    dm = DeviceModel(spec)
+    dm.set_input(x)
+    ctx = P.Context(0, P.config(packaging=2, graph=1, branches=1))
+    ctx.load_model(dm.graph)
+    s = torch.cuda.current_stream().cuda_stream
+    for _ in range(2):
+        ctx.infer(s)
+    ctx.sync()
+    (in_name, _, _), = spec["inputs"]
+    ref = [dm.t[o].cpu().clone() for o in spec["outputs"]]
+    in_cpu = dm.t[in_name].cpu().clone()
+    for pin in (True, False, True, True):
+        in_h = in_cpu.pin_memory() if pin else in_cpu.clone()
+        outs = [torch.zeros_like(r).pin_memory() if pin else torch.zeros_like(r) for r in ref]
+        ctx.infer_host([in_h.data_ptr()], [o.data_ptr() for o in outs], s)
+        for o, r in zip(outs, ref):
+            assert torch.equal(o.view(torch.int16) if o.dtype == torch.bfloat16 else o,
+                               r.view(torch.int16) if r.dtype == torch.bfloat16 else r), (name, pin)
+    for o in spec["outputs"]:
+        dm.t[o].zero_()
+    ctx.infer(s)                      # NULL buffers: the device tensors again
+    ctx.sync()
+    for o, r in zip(spec["outputs"], ref):
+        assert torch.equal(dm.t[o].cpu().view(torch.int16), r.view(torch.int16))
+    ctx.close()
