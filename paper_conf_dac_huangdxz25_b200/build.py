@@ -71,14 +71,18 @@ KERNELS = ["pask_layout", "pask_conv_igemm", "pask_conv_1x1", "pask_conv_dw", "p
 # The CNN variants also drop softmax's register-resident row path (their one
 # softmax row of 10 / 1000 classes takes the two-pass loop: same arithmetic,
 # bitwise equal) -- PASK_SOFTMAX_REG.
-FAMILY_VARIANTS = {"pask_families_tf": (0x30, 0x17), "pask_families_cnnf": (0xd5, 0x41),
+FAMILY_VARIANTS = {"pask_families_tf": (0x30, 0x17), "pask_families_cnng": (0x55, 0x21),
+                   "pask_families_cnnf": (0xd5, 0x41),
                    "pask_families_dwg": (0x5b, 0x25),
                    "pask_families_cnn": (0x55, 0x61), "pask_families_dw": (0x5f, 0x7f),
                    "pask_families": (0xff, 0x7f)}
-# (cnnf: a CNN whose narrow stem is folded (D16): the layout's fold path, memory
+# (cnng: a small CNN whose contractions all take the gather (and split-K), no
+# TMA im2col -- the tiny CNN;
+#  cnnf: a CNN whose narrow stem is folded (D16): the layout's fold path, memory
 # bit 7, and no cp.async gather -- ResNet-50; only cnnf and the full variant
 # carry the fold path)
-FAMILY_SOFTMAX_REG = {"pask_families_tf": 1, "pask_families_cnnf": 0, "pask_families_dwg": 0,
+FAMILY_SOFTMAX_REG = {"pask_families_tf": 1, "pask_families_cnng": 0, "pask_families_cnnf": 0,
+                      "pask_families_dwg": 0,
                       "pask_families_cnn": 0, "pask_families_dw": 1, "pask_families": 1}
 # Packaging 3 comes in the same variants: pask_single_<v> has the cases and paths
 # of pask_families_<v> behind the one entry pask_all (pask_single: everything).

@@ -242,7 +242,7 @@ def test_branches_issue_side_nodes_after_their_producer(name):
 
 
 @pytest.mark.parametrize("packaging", [2, 3])
-@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnn"), ("resnet50", "cnnf"), ("mobilenet_v2", "dwg"),
+@pytest.mark.parametrize("name,variant", [("tiny_cnn", "cnng"), ("resnet50", "cnnf"), ("mobilenet_v2", "dwg"),
                                           ("bert_base", "tf"), ("bert_base_fa", "tf")])
 def test_family_variant_covers_the_plan(name, variant, packaging):
     """Packaging 2 (D8): the families object is loaded in the smallest
