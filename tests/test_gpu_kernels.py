@@ -114,7 +114,30 @@ def test_stem_fold(case):
     spec = b.spec()
     from paper_conf_dac_huangdxz25_b200.model import DeviceModel
     assert DeviceModel(spec, alloc=False).ws_bytes > 0, "fold not taken"
-    _check_spec(spec)
+    xin = make_input(spec, 0)
+    dm, ctx, _ = run_model(spec, xin)
+    errs = teacher_forced_errors(dm, spec, xin)
+    ctx.close()
+    assert all(e <= TOL for _, _, e in errs), errs
+    # the workspace holds exactly the folded input and regrouped weights of the
+    # first conv reading the layout output (D16), restated from the
+    # formula in tests/stem_fold_ref.py: bit-exact (bf16 copies, zeros)
+    from .stem_fold_ref import fold_geometry, fold_input, fold_weights
+
+    def bits(a):
+        return (np.asarray(a, np.float64).astype(np.float32).view(np.uint32) >> 16).astype(np.uint16)
+
+    conv = next(L for L in spec["layers"] if L["op"] == "conv")
+    _, q, r2, t_rows = fold_geometry(h, w, c, r, r, (st, st), (pd, pd))
+    ws = dm.ws.cpu().numpy()
+    ybytes = n * t_rows * q * 64 * 2
+    y_ws = ws[:ybytes].view(np.uint16).reshape(n, t_rows, q, 64)
+    y_exp = bits(fold_input(O.bf16_rne(np.asarray(xin, np.float64)), r, r, (st, st), (pd, pd)).transpose(0, 2, 3, 1))
+    np.testing.assert_array_equal(y_ws, y_exp)
+    woff = (ybytes + 255) // 256 * 256
+    w_ws = ws[woff:woff + k * r2 * 64 * 2].view(np.uint16).reshape(k, r2, 64)
+    w_exp = bits(fold_weights(np.asarray(conv["w"], np.float64), (st, st))[..., 0].transpose(0, 2, 1))
+    np.testing.assert_array_equal(w_ws, w_exp)
 
 
 _NOFOLD_CHILD = r"""
