@@ -415,10 +415,11 @@ def main():
         try:
             with cs.Keeper(image, cfg):
                 main_cold = cold_block(cs, image, cfg, args.cold_samples, args.timeline_samples, False)
-                main_cold["cold_no_prefault"] = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1},
-                                                                       args.ablation_samples))
-                main_cold["cold_no_prime"] = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1},
-                                                                    args.ablation_samples))
+                if args.ablation_samples > 0:
+                    main_cold["cold_no_prefault"] = cs.summarize(cs.sample(image, {**cfg, "no_prefault": 1},
+                                                                           args.ablation_samples))
+                    main_cold["cold_no_prime"] = cs.summarize(cs.sample(image, {**cfg, "no_prime": 1},
+                                                                        args.ablation_samples))
                 py = [cs.run_py_child(args.model, cfg, args.batch) for _ in range(args.py_cold_samples)]
                 main_cold["cold_python_process"] = cs.summarize(py) if py else None
                 if not args.no_configs and args.batch == 1:
@@ -683,13 +684,13 @@ def main():
     # this process's hot numbers for the main config
     headline = {}
     if main_cold is not None:
-        c, nopf, nopr = main_cold["cold"], main_cold["cold_no_prefault"], main_cold["cold_no_prime"]
+        c, nopf, nopr = main_cold["cold"], main_cold.get("cold_no_prefault"), main_cold.get("cold_no_prime")
         pyc = main_cold["cold_python_process"]
+        ms2 = lambda d: [round(d["median_us"] / 1e3, 3), round(d["p90_us"] / 1e3, 3)] if d else None  # noqa: E731
         headline[args.model] = headline_entry(
             c["median_us"] / 1e3, c["p90_us"] / 1e3, c["n"], hot_max, direct_max, main_cold["breakdown"],
             c["kernels_loaded"], main_cold["launches"],
-            {"nopf_ms": [round(nopf["median_us"] / 1e3, 3), round(nopf["p90_us"] / 1e3, 3)],
-             "noprime_ms": [round(nopr["median_us"] / 1e3, 3), round(nopr["p90_us"] / 1e3, 3)],
+            {"nopf_ms": ms2(nopf), "noprime_ms": ms2(nopr),
              "py_ms": ([round(pyc["median_us"] / 1e3, 3), round(pyc["p90_us"] / 1e3, 3), pyc["n"]]
                        if pyc else None)})
         for m, blk in configs_detail.items():
